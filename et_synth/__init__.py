@@ -1,0 +1,191 @@
+"""Seeded synthetic inputs shared by the oracle, the tests and bench.py.
+
+This module holds NO arithmetic of the E.T. method (no pruning, no attention,
+no projection): it only draws random numbers and rounds them to the storage
+dtype, so that the CPU oracle (`oracle/`) and the CUDA path
+(`paper_conf_sc_chenhplg0d021_b200`) consume bit-identical inputs.  Neither
+side imports the other; both import this.
+
+Recipe:
+  * generator: numpy.random.Generator(PCG64(seed)); draws are float32, then
+    rounded to the storage dtype on the host (round-to-nearest-even);
+  * X ~ N(0, 1) of shape [B, S, d], seed 1000;
+  * layer l, matrix k uses seed 2000 + 16*l + k:
+      W_Q, W_K ~ N(0, 0.05^2)  (score std ~2 at d=768, d_k=64 so softmax is
+                                non-trivial; BERT's 0.02 init gives a nearly
+                                uniform softmax);
+      W_V, W_O, W_1, W_2 ~ N(0, 0.02^2); every bias ~ N(0, 0.02^2);
+      gamma = 1 + N(0, 0.05^2); beta ~ N(0, 0.02^2);
+  * lengths: throughput runs use all S; parity runs draw U{ceil(S/4)..S} with
+    seed 3000 and force lengths[0] = S and lengths[1] = 1 (padding edge cases).
+
+Weights follow the paper's convention W = [out, in] (Q = X . W_Q^T, PAPER.md
+line 68, §2.1).
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+
+import numpy as np
+
+# --------------------------------------------------------------------------
+# workload configurations (BASELINE.json "configs")
+# --------------------------------------------------------------------------
+
+
+@dataclasses.dataclass(frozen=True)
+class Config:
+    name: str
+    layers: int
+    heads: int
+    d_model: int
+    d_ff: int
+    seq_len: int
+    batch: int
+    ratio: float
+    scheme: str          # "tile" (all six matrices tile-pruned) or "attention-aware" (W_V row)
+    dtype: str           # "fp16" | "bf16" | "fp32"
+    act: str             # "gelu" | "relu"
+    ln_eps: float
+    causal: bool
+    attn_mode: str = "auto"   # "auto" | "short" | "long"
+
+    @property
+    def d_k(self) -> int:
+        return self.d_model // self.heads
+
+    @property
+    def tokens(self) -> int:
+        return self.batch * self.seq_len
+
+    def with_(self, **kw) -> "Config":
+        return dataclasses.replace(self, **kw)
+
+
+CONFIGS = {
+    # configs[0]: single layer, 1 head, d=64, S=16, B=1, 50% tile pruning, FP32
+    "C1": Config("C1", 1, 1, 64, 256, 16, 1, 0.5, "tile", "fp32", "gelu", 1e-12, False),
+    # configs[1]: 4-head Transformer encoder d=512, S=128, B=1, 80% (Fig. 1)
+    "C2": Config("C2", 1, 4, 512, 2048, 128, 1, 0.8, "attention-aware", "fp16", "relu", 1e-5, True),
+    # configs[2]: BERT-base, S=128, B=32, 80% tile pruning, FP16 (the headline)
+    "C3": Config("C3", 12, 12, 768, 3072, 128, 32, 0.8, "tile", "fp16", "gelu", 1e-12, False),
+    # configs[3]: DistilBERT, S=512, B=64, row pruning (attention-aware), long-sequence operator
+    "C4": Config("C4", 6, 12, 768, 3072, 512, 64, 0.8, "attention-aware", "fp16", "gelu", 1e-12, False,
+                 "long"),
+    # configs[4]: BERT-base, S=2048, B=256, tile pruning, batch-sharded over 1/2/4/8 GPUs
+    "C5": Config("C5", 12, 12, 768, 3072, 2048, 256, 0.8, "tile", "fp16", "gelu", 1e-12, False, "long"),
+}
+
+MATRICES = ("wq", "wk", "wv", "wo", "w1", "w2")
+
+
+def matrix_pattern(scheme: str, name: str) -> str:
+    """Pruning pattern per matrix (Fig. 3(a) caption, line 317 §5.3).
+
+    "tile": every matrix tensor-tile pruned.  "attention-aware": W_V row pruned,
+    all other weights tile pruned.  "none": dense.  This is a table lookup, not
+    method arithmetic.
+    """
+    if scheme == "none":
+        return "none"
+    if scheme == "tile":
+        return "tile"
+    if scheme == "attention-aware":
+        return "row" if name == "wv" else "tile"
+    raise ValueError(scheme)
+
+
+# --------------------------------------------------------------------------
+# rounding to the storage dtype (input quantisation only)
+# --------------------------------------------------------------------------
+
+
+def round_bf16(x: np.ndarray) -> np.ndarray:
+    """Round float32 values to the nearest bfloat16 (ties to even); returns float32."""
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    u = x.view(np.uint32).astype(np.uint64)
+    lsb = (u >> 16) & 1
+    u = (u + 0x7FFF + lsb) & 0xFFFF0000
+    return u.astype(np.uint32).view(np.float32)
+
+
+def to_storage(x: np.ndarray, dtype: str) -> np.ndarray:
+    """Round to the storage dtype and return float32 values that are exactly representable in it."""
+    x = np.asarray(x, dtype=np.float32)
+    if dtype == "fp32":
+        return x.copy()
+    if dtype == "fp16":
+        return x.astype(np.float16).astype(np.float32)
+    if dtype == "bf16":
+        return round_bf16(x)
+    raise ValueError(dtype)
+
+
+def _rng(seed: int) -> np.random.Generator:
+    return np.random.Generator(np.random.PCG64(seed))
+
+
+def _normal(seed: int, shape, std: float, mean: float = 0.0) -> np.ndarray:
+    g = _rng(seed)
+    return (mean + std * g.standard_normal(shape, dtype=np.float32)).astype(np.float32)
+
+
+# --------------------------------------------------------------------------
+# generators
+# --------------------------------------------------------------------------
+
+
+def make_x(cfg: Config, dtype: str | None = None, seed: int = 1000) -> np.ndarray:
+    """Token embeddings X ~ N(0,1), shape [B, S, d], rounded to the storage dtype."""
+    dt = dtype or cfg.dtype
+    return to_storage(_normal(seed, (cfg.batch, cfg.seq_len, cfg.d_model), 1.0), dt)
+
+
+def make_layer(cfg: Config, layer: int, dtype: str | None = None) -> dict:
+    """Random-init weights of one encoder layer (float32 arrays holding storage-dtype values).
+
+    Shapes: wq/wk/wv/wo [d, d]; w1 [d_ff, d]; w2 [d, d_ff]; biases [out];
+    ln1_g/ln1_b/ln2_g/ln2_b [d].  LayerNorm parameters are kept in float32.
+    """
+    dt = dtype or cfg.dtype
+    d, f = cfg.d_model, cfg.d_ff
+    s0 = 2000 + 16 * layer
+    out = {
+        "wq": to_storage(_normal(s0 + 0, (d, d), 0.05), dt),
+        "wk": to_storage(_normal(s0 + 1, (d, d), 0.05), dt),
+        "wv": to_storage(_normal(s0 + 2, (d, d), 0.02), dt),
+        "wo": to_storage(_normal(s0 + 3, (d, d), 0.02), dt),
+        "w1": to_storage(_normal(s0 + 4, (f, d), 0.02), dt),
+        "w2": to_storage(_normal(s0 + 5, (d, f), 0.02), dt),
+        "bq": to_storage(_normal(s0 + 6, (d,), 0.02), dt),
+        "bk": to_storage(_normal(s0 + 7, (d,), 0.02), dt),
+        "bv": to_storage(_normal(s0 + 8, (d,), 0.02), dt),
+        "bo": to_storage(_normal(s0 + 9, (d,), 0.02), dt),
+        "b1": to_storage(_normal(s0 + 10, (f,), 0.02), dt),
+        "b2": to_storage(_normal(s0 + 11, (d,), 0.02), dt),
+        "ln1_g": _normal(s0 + 12, (d,), 0.05, 1.0),
+        "ln1_b": _normal(s0 + 13, (d,), 0.02),
+        "ln2_g": _normal(s0 + 14, (d,), 0.05, 1.0),
+        "ln2_b": _normal(s0 + 15, (d,), 0.02),
+    }
+    return out
+
+
+def make_lengths(cfg: Config, ragged: bool = True, seed: int = 3000) -> np.ndarray:
+    """Valid lengths per sequence (int32 [B]); ragged draws U{ceil(S/4)..S}."""
+    S, B = cfg.seq_len, cfg.batch
+    if not ragged:
+        return np.full((B,), S, dtype=np.int32)
+    g = _rng(seed)
+    lo = max(1, math.ceil(S / 4))
+    lens = g.integers(lo, S + 1, size=(B,)).astype(np.int32)
+    lens[0] = S
+    if B > 1:
+        lens[1] = 1
+    return lens
+
+
+def make_matrix(seed: int, shape, std: float, dtype: str) -> np.ndarray:
+    """A single random matrix in the storage dtype (used by pack / GEMM tests)."""
+    return to_storage(_normal(seed, shape, std), dtype)
