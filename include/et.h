@@ -1,0 +1,229 @@
+/*
+ * et.h — C ABI of the B200-native (sm_100a) hot path of E.T. (Chen et al., SC'21,
+ * "E.T.: Re-Thinking Self-Attention for Transformer Models on GPUs"; PAPER.md below).
+ *
+ * The library computes the forward pass of a post-LN Transformer encoder whose
+ * Q/K/V/O and FFN weights are pruned with tensor tiles (§4.2) or
+ * rows (line 171, §4.1), with the on-the-fly attention operator (line 99-113, §3.1) in a
+ * short- and a long-sequence form (line 133-147, §3.2) and the scale moved before Q.K^T
+ * (line 159, §3.3).
+ *
+ * Conventions (all entry points):
+ *   - Every function returns et_status; no exception crosses the ABI.  et_last_error() returns
+ *     a thread-local message describing the last failure of the calling thread.
+ *   - All arguments are validated before anything is launched.  Launch errors are reported as
+ *     ET_ERR_CUDA; asynchronous device faults surface at the caller's next synchronisation.
+ *   - Device pointers are plain CUDA device pointers allocated BY THE CALLER (the library never
+ *     allocates device memory).  Work is enqueued on the caller's stream; nothing synchronises
+ *     the device except et_prune_pack (documented below).  The forward entry points are
+ *     CUDA-graph capturable.
+ *   - Matrices are row-major.  Weights are [out, in]; Y = X . W^T (§2.1).
+ *   - Activations X / out are [batch * seq_len, d_model]; token t = b * seq_len + s.
+ *   - Tensor-core operands must be 16-byte aligned (TMA); ET_ERR_INVALID_ARG otherwise.
+ *   - Thread-safe and reentrant: no mutable global state beyond the error string and a
+ *     lazily-initialised, read-only kernel attribute cache.
+ */
+#ifndef ET_H_
+#define ET_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  ET_OK = 0,
+  ET_ERR_INVALID_ARG = 1,  /* bad shape / pointer / enum / alignment */
+  ET_ERR_UNSUPPORTED = 2,  /* valid request this build does not implement (message says which) */
+  ET_ERR_WORKSPACE = 3,    /* workspace too small (query the *_workspace_size function) */
+  ET_ERR_CUDA = 4,         /* a CUDA runtime / launch error */
+  ET_ERR_NCCL = 5,         /* reserved for the head-parallel collective */
+  ET_ERR_INTERNAL = 6
+} et_status;
+
+typedef enum { ET_FP16 = 0, ET_BF16 = 1, ET_FP32 = 2 } et_dtype;
+
+/* Pruning patterns (§4.1-4.2; attention-aware assignment line 107, 317). */
+typedef enum { ET_PRUNE_NONE = 0, ET_PRUNE_TILE = 1, ET_PRUNE_ROW = 2, ET_PRUNE_COL = 3 } et_pattern;
+
+/* Attention operator form (§3.2, switch at a length threshold line 244). */
+typedef enum { ET_ATTN_AUTO = 0, ET_ATTN_SHORT = 1, ET_ATTN_LONG = 2 } et_attn_mode;
+
+/* FFN activation ("an activation layer"; GELU(erf) for BERT, ReLU otherwise). */
+typedef enum { ET_ACT_GELU_ERF = 0, ET_ACT_RELU = 1 } et_act;
+
+const char* et_last_error(void);
+const char* et_version(void);
+
+/* ------------------------------------------------------------------------------------------
+ * Packed pruned weight.  Produced by et_prune_pack; consumed by the forward entry points.
+ * All pointer fields are device memory allocated by the caller with the sizes returned by
+ * et_prune_pack_query.  Fields:
+ *   pattern, dtype, rows (= out), cols (= in), tile_r, tile_c       as requested
+ *   group_rows   ROW only: rows are padded per group of group_rows original rows (one attention
+ *                head: d_k) to a multiple of 16 so that every head's V width is MMA-aligned
+ *                (reading C-5); 0 = one group.
+ *   nnz          kept units: tiles (TILE) / rows (ROW) / columns (COL); filled by et_prune_pack
+ *   rows_padded  ROW: packed row count (sum over groups of round_up(kept_g, 16)); TILE: rows
+ *   mask         bitmap over units, ceil(T/32) uint32 words, unit t at bit t%32 of word t/32,
+ *                1 = kept.  TILE: t = i*(cols/tile_c) + j.  ROW: t = row.  BIT-EXACT contract.
+ *   idx          TILE: CSR col_idx[nnz] (ascending within each tile row).  ROW/COL: kept
+ *                row/column indices [nnz], ascending.  BIT-EXACT contract.
+ *   row_ptr      TILE: CSR row_ptr[rows/tile_r + 1] (BIT-EXACT contract).  ROW: the uniform
+ *                tile CSR of the dense packed matrix [rows_padded/16 + 1].
+ *   tile_col     tile column of every packed tile, in values order [ntiles].
+ *   row_map      ROW: [rows_padded] original row of each packed row, -1 for padding.  TILE: unused.
+ *   kparts       number of K parts of at most 768 columns (48 tile columns) each: ceil(cols/768).
+ *   part_row_ptr [kparts][tile_rows + 1]: packed tiles of K part z and tile row i are
+ *                values[part_row_ptr[z][i] .. part_row_ptr[z][i+1]) (for kparts == 1 this is the
+ *                CSR row_ptr).  Lets split-K GEMM CTAs stream their tiles contiguously.
+ *   values       the kept 16x16 tiles in (K part, tile row, tile column) order, each 512 bytes (16-bit dtypes) in the
+ *                tcgen05 K-major no-swizzle core-matrix layout: element (n, k) of a tile at byte
+ *                (n/8)*256 + (k/8)*128 + (n%8)*16 + (k%8)*2.  Only for tile_r = tile_c = 16 and
+ *                FP16/BF16; may be NULL otherwise (mask / index only).
+ * ------------------------------------------------------------------------------------------ */
+typedef struct {
+  et_pattern pattern;
+  et_dtype dtype;
+  int32_t rows, cols, tile_r, tile_c, group_rows;
+  int32_t nnz;
+  int32_t rows_padded;
+  int32_t ntiles;   /* number of packed tiles (TILE: nnz; ROW: rows_padded/16 * cols/16) */
+  int32_t kparts;
+  uint32_t* mask;
+  int32_t* idx;
+  int32_t* row_ptr;
+  int32_t* tile_col;     /* in values order */
+  int32_t* row_map;
+  int32_t* part_row_ptr;
+  void* values;
+} et_packed_weight;
+
+/* Host-only size query (no CUDA call).  Returns worst-case buffer sizes for et_prune_pack.
+ *   ratio in [0, 1]; n_prune = floor(ratio * T + 0.5) units are pruned (reading C-2).
+ *   rows % tile_r == 0 and cols % tile_c == 0 required (TILE), else ET_ERR_INVALID_ARG.
+ *   nnz_out: exact kept count (= T - n_prune, or popcount of mask_in when host_mask_in given).
+ * Any output pointer may be NULL. */
+et_status et_prune_pack_query(int32_t rows, int32_t cols, et_dtype dtype, et_pattern pattern, double ratio,
+                              int32_t tile_r, int32_t tile_c, int32_t group_rows, const uint32_t* host_mask_in,
+                              int32_t* nnz_out, size_t* mask_bytes, size_t* idx_bytes, size_t* rowptr_bytes,
+                              size_t* tilecol_bytes, size_t* rowmap_bytes, size_t* partrowptr_bytes,
+                              size_t* values_bytes, size_t* workspace_bytes);
+
+/* Prune and pack one weight matrix (§4.2 step (v) 1-4; line 171 §4.1):
+ * squared l2 norm per unit accumulated in FP64 in a fixed order (tile: a outer, b inner),
+ * rank by (score, linear index), prune the lowest n_prune, emit mask / index / packed values.
+ *   W_dev        device [rows, cols] in dtype
+ *   mask_in_dev  optional device bitmap (same format as out->mask) fixing the kept set
+ *   out          caller-filled buffers (sizes from the query); on return out->nnz,
+ *                out->rows_padded and out->ntiles are set.
+ * Deterministic.  SYNCHRONISES `stream` before returning (it is an offline, once-per-weight
+ * step; the counts are needed on the host). */
+et_status et_prune_pack(const void* W_dev, int32_t rows, int32_t cols, et_dtype dtype, et_pattern pattern,
+                        double ratio, int32_t tile_r, int32_t tile_c, int32_t group_rows,
+                        const uint32_t* mask_in_dev, et_packed_weight* out, void* workspace,
+                        size_t workspace_bytes, void* stream);
+
+/* Expand a packed weight back to a dense [rows, cols] matrix W' = mask (.) W (test hook; used
+ * to check values bit-exactly).  dense_out: device [rows, cols] in the packed dtype. */
+et_status et_unpack(const et_packed_weight* w, void* dense_out, void* stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Tile-sparse linear layer (test hook + building block):
+ *   Y[M, N] = epilogue(X[M, K] . W'^T + b)         N = w->rows (ROW: rows_padded), K = w->cols
+ * Skips pruned tiles (one tcgen05.mma per kept 16x16 tile).  epilogue:
+ *   ET_EPI_BIAS        Y = acc + b                              (out dtype = X dtype)
+ *   ET_EPI_BIAS_SCALE  Y = (acc + b) * scale for columns < scale_cols, acc + b otherwise
+ *                      (the 1/sqrt(d_k) of Q moved before Q.K^T, line 159 §3.3)
+ *   ET_EPI_BIAS_GELU / ET_EPI_BIAS_RELU  Y = act(acc + b)
+ *   ET_EPI_F32         Y = acc (fp32, no bias) — partial sums for a LayerNorm epilogue
+ * X: [M, K] fp16/bf16, M % 128 == 0 not required (rows are masked).  b: [N] in X's dtype or NULL. */
+typedef enum { ET_EPI_BIAS = 0, ET_EPI_BIAS_SCALE = 1, ET_EPI_BIAS_GELU = 2, ET_EPI_BIAS_RELU = 3, ET_EPI_F32 = 4 } et_epilogue;
+
+et_status et_linear_fwd(const et_packed_weight* w, const void* X, int32_t M, const void* bias, et_epilogue epi,
+                        float scale, int32_t scale_cols, void* Y, void* stream);
+
+/* Residual + LayerNorm: out = LN(sum_p part[p] + bias + resid) * gamma + beta
+ *   part: nparts x [M, N] fp32; bias [N] (dtype) or NULL; resid [M, N] in resid_dtype or NULL;
+ *   gamma/beta fp32 [N]; out_act [M, N] in act_dtype (GEMM operand copy) and/or out_resid
+ *   [M, N] in resid_dtype (either may be NULL).  Biased variance (reading C-11). */
+et_status et_layernorm_fwd(const float* part, int32_t nparts, int32_t M, int32_t N, const void* bias,
+                           et_dtype dtype, const void* resid, et_dtype resid_dtype, const float* gamma,
+                           const float* beta, float eps, void* out_act, void* out_resid, void* stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Attention descriptor.
+ *   batch, seq_len, heads, d_model   problem statement (d_k = d_model / H)
+ *   dtype        storage dtype of activations and weights (FP16 / BF16)
+ *   lengths_dev  device int32 [batch], valid length per sequence, 1 <= len <= seq_len; keys
+ *                j >= len are masked (probability exactly 0, line 73; reading C-7).  NULL = all.
+ *   causal       nonzero: also mask j > i (the triangular mask of line 73)
+ *   mode         short / long / auto (auto: short while seq_len <= et_attn_short_max())
+ *   head_begin, head_end   head range computed by this call ([0, H) normally; a sub-range in
+ *                head-parallel mode, where `out` receives that range's W_O partial sum:
+ *                bias only if head_begin == 0, no residual/LN — Eq. 4).
+ * ------------------------------------------------------------------------------------------ */
+typedef struct {
+  int32_t batch, seq_len, heads, d_model;
+  et_dtype dtype;
+  const int32_t* lengths_dev;
+  int32_t causal;
+  et_attn_mode mode;
+  int32_t head_begin, head_end;
+} et_attn_desc;
+
+/* Largest seq_len served by the short (score row resident in TMEM) form. */
+int32_t et_attn_short_max(int32_t d_k);
+
+/* Attention core (steps 2-6 of Fig. 3(a)):
+ *   Z[:, h*dv : (h+1)*dv] = softmax(mask(Q_h . K_h^T * scale)) . V_h      for h in [head_begin, head_end)
+ * qkv: [batch*seq_len, ld_qkv] holding Q at column q_off + h*d_k, K at k_off + h*d_k and V at
+ * v_off + v_col[h] (v_col / v_width: device int32 [heads] or NULL for V laid out like Q, i.e.
+ * v_col[h] = h*d_k, v_width[h] = d_k).  `scale` multiplies the scores (pass 1 if Q was already
+ * scaled by 1/sqrt(d_k), the reordered form of line 159).  Z: [batch*seq_len, ld_z], head h
+ * written at column z_col[h] (NULL => h*d_k) — V widths padded to 16 with zero rows write
+ * zeros.  The seq x seq score matrix never leaves TMEM / registers. */
+et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld_qkv, int32_t q_off, int32_t k_off,
+                           int32_t v_off, const int32_t* v_col, const int32_t* v_width, float scale, void* Z,
+                           int32_t ld_z, const int32_t* z_col, void* stream);
+
+/* Self-attention block (Fig. 3(a) steps 1-7, Eq. 3-4):
+ *   out = SelfAttn(X)                  if ln_gamma == NULL
+ *   out = LN(X + SelfAttn(X))          otherwise (post-LN, line 75)
+ * wq, wk, wo: TILE (or NONE packed as all-kept TILE); wv: TILE or ROW (attention-aware,
+ * line 107/317).  Biases in dtype; ln params fp32.  X, out: [batch*seq_len, d_model] in dtype. */
+et_status et_attention_workspace_size(const et_attn_desc* desc, const et_packed_weight* wv, size_t* bytes);
+et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_packed_weight* wq,
+                           const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
+                           const void* bq, const void* bk, const void* bv, const void* bo, const float* ln_gamma,
+                           const float* ln_beta, float ln_eps, void* out, void* workspace, size_t ws_bytes,
+                           void* stream);
+
+/* One encoder layer's parameters.  Weights packed; biases in the storage dtype; LN fp32. */
+typedef struct {
+  et_packed_weight wq, wk, wv, wo, w1, w2;
+  const void *bq, *bk, *bv, *bo, *b1, *b2;
+  const float *ln1_g, *ln1_b, *ln2_g, *ln2_b;
+} et_layer;
+
+/* Post-LN encoder stack:  for each layer:
+ *   Y1 = LN(X + SelfAttn(X));  U = act(Y1 W1'^T + b1);  Y2 = LN(Y1 + U W2'^T + b2).
+ * X, out: [batch*seq_len, d_model] in resid_dtype (FP32, or equal to desc->dtype; reading C-22);
+ * GEMM operands in desc->dtype.  layers_host: host array of num_layers et_layer.  X and out
+ * may alias.  No host synchronisation; CUDA-graph capturable. */
+et_status et_encoder_workspace_size(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff,
+                                    et_dtype resid_dtype, const et_layer* layers_host, size_t* bytes);
+et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff, et_act act, float ln_eps,
+                         et_dtype resid_dtype, const et_layer* layers_host, const void* X, void* out,
+                         void* workspace, size_t ws_bytes, void* stream);
+
+/* Diagnostics (not part of the metric): tcgen05 probe (profiles/r01/M1_tcgen05_probe.md). */
+int et_diag_mma_probe(const void* A, const void* B, float* D, int N, int a_mode, int b_mode, int iters, int n_acc,
+                      int issue_mode, long long* cycles, int grid, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ET_H_ */

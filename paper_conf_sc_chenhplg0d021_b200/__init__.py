@@ -1,0 +1,234 @@
+"""Python binding of libet.so — the B200-native (sm_100a) hot path of E.T. (SC'21).
+
+Argument marshalling only: every step of the path runs in the CUDA kernels of libet.so
+(include/et.h).  PyTorch is used for device memory and streams; there is no CPU fallback:
+loading fails loudly if the library is missing, and every call raises on a non-OK status.
+
+Names follow the C ABI: prune_pack, unpack, linear_fwd, layernorm_fwd, attn_core_fwd,
+attention_fwd, encoder_fwd (+ the *_workspace_size queries).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.environ.get("ET_LIB_PATH") or os.path.join(_HERE, "libet.so")
+
+# enums (include/et.h)
+FP16, BF16, FP32 = 0, 1, 2
+PRUNE_NONE, PRUNE_TILE, PRUNE_ROW, PRUNE_COL = 0, 1, 2, 3
+ATTN_AUTO, ATTN_SHORT, ATTN_LONG = 0, 1, 2
+ACT_GELU_ERF, ACT_RELU = 0, 1
+EPI_BIAS, EPI_BIAS_SCALE, EPI_BIAS_GELU, EPI_BIAS_RELU, EPI_F32 = 0, 1, 2, 3, 4
+
+_DT = {"fp16": FP16, "bf16": BF16, "fp32": FP32}
+_TORCH_DT = {FP16: torch.float16, BF16: torch.bfloat16, FP32: torch.float32}
+_PAT = {"none": PRUNE_NONE, "tile": PRUNE_TILE, "row": PRUNE_ROW, "col": PRUNE_COL}
+_MODE = {"auto": ATTN_AUTO, "short": ATTN_SHORT, "long": ATTN_LONG}
+_ACT = {"gelu": ACT_GELU_ERF, "relu": ACT_RELU}
+
+
+class EtError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"et status {status}: {msg}")
+        self.status = status
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_sc_chenhplg0d021_b200.build` "
+                          "(there is no CPU fallback)")
+    return ctypes.CDLL(LIB_PATH)
+
+
+_lib = _load()
+_vp, _i32, _sz, _f32, _f64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_size_t, ctypes.c_float, ctypes.c_double
+
+
+class PackedWeightC(ctypes.Structure):
+    _fields_ = [("pattern", ctypes.c_int), ("dtype", ctypes.c_int), ("rows", _i32), ("cols", _i32),
+                ("tile_r", _i32), ("tile_c", _i32), ("group_rows", _i32), ("nnz", _i32), ("rows_padded", _i32),
+                ("ntiles", _i32), ("kparts", _i32), ("mask", _vp), ("idx", _vp), ("row_ptr", _vp),
+                ("tile_col", _vp), ("row_map", _vp), ("part_row_ptr", _vp), ("values", _vp)]
+
+
+class AttnDescC(ctypes.Structure):
+    _fields_ = [("batch", _i32), ("seq_len", _i32), ("heads", _i32), ("d_model", _i32), ("dtype", ctypes.c_int),
+                ("lengths_dev", _vp), ("causal", _i32), ("mode", ctypes.c_int), ("head_begin", _i32),
+                ("head_end", _i32)]
+
+
+class LayerC(ctypes.Structure):
+    _fields_ = [("wq", PackedWeightC), ("wk", PackedWeightC), ("wv", PackedWeightC), ("wo", PackedWeightC),
+                ("w1", PackedWeightC), ("w2", PackedWeightC), ("bq", _vp), ("bk", _vp), ("bv", _vp), ("bo", _vp),
+                ("b1", _vp), ("b2", _vp), ("ln1_g", _vp), ("ln1_b", _vp), ("ln2_g", _vp), ("ln2_b", _vp)]
+
+
+def _sig(name, res, args):
+    f = getattr(_lib, name)
+    f.restype = res
+    f.argtypes = args
+    return f
+
+
+_lib.et_last_error.restype = ctypes.c_char_p
+_lib.et_version.restype = ctypes.c_char_p
+_sz_p = ctypes.POINTER(_sz)
+_q = _sig("et_prune_pack_query", ctypes.c_int,
+          [_i32, _i32, ctypes.c_int, ctypes.c_int, _f64, _i32, _i32, _i32, _vp, ctypes.POINTER(_i32)] + [_sz_p] * 8)
+_pack = _sig("et_prune_pack", ctypes.c_int,
+             [_vp, _i32, _i32, ctypes.c_int, ctypes.c_int, _f64, _i32, _i32, _i32, _vp,
+              ctypes.POINTER(PackedWeightC), _vp, _sz, _vp])
+_unpack = _sig("et_unpack", ctypes.c_int, [ctypes.POINTER(PackedWeightC), _vp, _vp])
+_linear = _sig("et_linear_fwd", ctypes.c_int,
+               [ctypes.POINTER(PackedWeightC), _vp, _i32, _vp, ctypes.c_int, _f32, _i32, _vp, _vp])
+_ln = _sig("et_layernorm_fwd", ctypes.c_int,
+           [_vp, _i32, _i32, _i32, _vp, ctypes.c_int, _vp, ctypes.c_int, _vp, _vp, _f32, _vp, _vp, _vp])
+_short_max = _sig("et_attn_short_max", _i32, [_i32])
+
+SYMBOLS = ["et_last_error", "et_version", "et_prune_pack_query", "et_prune_pack", "et_unpack", "et_linear_fwd",
+           "et_layernorm_fwd", "et_attn_short_max", "et_attn_core_fwd", "et_attention_workspace_size",
+           "et_attention_fwd", "et_encoder_workspace_size", "et_encoder_fwd", "et_diag_mma_probe"]
+
+
+def _check(st: int):
+    if st != 0:
+        raise EtError(st, _lib.et_last_error().decode())
+
+
+def version() -> str:
+    return _lib.et_version().decode()
+
+
+def _stream(stream=None) -> int:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+def _ptr(t):
+    return None if t is None else t.data_ptr()
+
+
+def dtype_code(dt) -> int:
+    if isinstance(dt, int):
+        return dt
+    if isinstance(dt, torch.dtype):
+        return {torch.float16: FP16, torch.bfloat16: BF16, torch.float32: FP32}[dt]
+    return _DT[dt]
+
+
+def torch_dtype(code) -> torch.dtype:
+    return _TORCH_DT[dtype_code(code)]
+
+
+# ------------------------------------------------------------------------------------------ packing
+class Packed:
+    """A packed pruned weight: the device buffers (torch tensors) + the C struct pointing at them."""
+
+    def __init__(self, c: PackedWeightC, bufs: dict):
+        self.c = c
+        self.bufs = bufs
+
+    @property
+    def nnz(self):
+        return self.c.nnz
+
+    @property
+    def rows_padded(self):
+        return self.c.rows_padded
+
+    def mask(self):
+        return self.bufs["mask"]
+
+    def units(self):
+        c = self.c
+        if c.pattern == PRUNE_TILE:
+            return (c.rows // c.tile_r) * (c.cols // c.tile_c)
+        return c.rows if c.pattern == PRUNE_ROW else c.cols
+
+    def csr(self):
+        """(row_ptr, col_idx) of a TILE weight (the bit-exact contract)."""
+        p = self.c.rows // self.c.tile_r
+        return self.bufs["row_ptr"][:p + 1], self.bufs["idx"][:self.c.nnz]
+
+    def kept_index(self):
+        return self.bufs["idx"][:self.c.nnz]
+
+
+def prune_pack(W: torch.Tensor, pattern: str = "tile", ratio: float = 0.8, tile=(16, 16), group_rows: int = 0,
+               mask_in: torch.Tensor | None = None, stream=None) -> Packed:
+    """et_prune_pack: prune and pack a device weight W [rows, cols] (fp16 / bf16 / fp32)."""
+    assert W.is_cuda and W.dim() == 2 and W.is_contiguous()
+    rows, cols = W.shape
+    dt = dtype_code(W.dtype)
+    pat = _PAT[pattern] if isinstance(pattern, str) else pattern
+    sizes = [_sz() for _ in range(8)]
+    nnz = _i32()
+    _check(_q(rows, cols, dt, pat, ratio, tile[0], tile[1], group_rows, None, ctypes.byref(nnz),
+              *[ctypes.byref(s) for s in sizes]))
+    names = ["mask", "idx", "row_ptr", "tile_col", "row_map", "part_row_ptr", "values", "ws"]
+    dev = W.device
+    bufs = {}
+    for n, s in zip(names, sizes):
+        nb = max(int(s.value), 16)
+        bufs[n] = torch.empty(((nb + 15) // 16) * 16, dtype=torch.uint8, device=dev)
+    c = PackedWeightC()
+    c.mask = bufs["mask"].data_ptr()
+    c.idx = bufs["idx"].data_ptr()
+    c.row_ptr = bufs["row_ptr"].data_ptr()
+    c.tile_col = bufs["tile_col"].data_ptr()
+    c.row_map = bufs["row_map"].data_ptr()
+    c.part_row_ptr = bufs["part_row_ptr"].data_ptr()
+    c.values = bufs["values"].data_ptr() if sizes[6].value > 0 else None
+    _check(_pack(W.data_ptr(), rows, cols, dt, pat, ratio, tile[0], tile[1], group_rows,
+                 _ptr(mask_in), ctypes.byref(c), bufs["ws"].data_ptr(), bufs["ws"].numel(), _stream(stream)))
+    del bufs["ws"]
+    views = {
+        "mask": bufs["mask"].view(torch.int32),
+        "idx": bufs["idx"].view(torch.int32),
+        "row_ptr": bufs["row_ptr"].view(torch.int32),
+        "tile_col": bufs["tile_col"].view(torch.int32),
+        "row_map": bufs["row_map"].view(torch.int32),
+        "part_row_ptr": bufs["part_row_ptr"].view(torch.int32),
+        "values": bufs["values"],
+    }
+    return Packed(c, views)
+
+
+def unpack(w: Packed, stream=None) -> torch.Tensor:
+    """et_unpack: dense W' = mask (.) W [rows, cols] from the packed values."""
+    out = torch.empty(w.c.rows, w.c.cols, dtype=torch_dtype(w.c.dtype), device=w.bufs["values"].device)
+    _check(_unpack(ctypes.byref(w.c), out.data_ptr(), _stream(stream)))
+    return out
+
+
+# ------------------------------------------------------------------------------------------ linear / LN
+def linear_fwd(w: Packed, X: torch.Tensor, bias: torch.Tensor | None = None, epi: int = EPI_BIAS,
+               scale: float = 1.0, scale_cols: int = 0, out: torch.Tensor | None = None, stream=None):
+    """et_linear_fwd: Y = epilogue(X . W'^T + b) skipping pruned tiles."""
+    M = X.shape[0]
+    N = w.c.rows if w.c.pattern == PRUNE_TILE else w.c.rows_padded
+    if out is None:
+        if epi == EPI_F32:
+            out = torch.empty(w.c.kparts, M, N, dtype=torch.float32, device=X.device)
+        else:
+            out = torch.empty(M, N, dtype=X.dtype, device=X.device)
+    _check(_linear(ctypes.byref(w.c), X.data_ptr(), M, _ptr(bias), epi, scale, scale_cols, out.data_ptr(),
+                   _stream(stream)))
+    return out
+
+
+def layernorm_fwd(part: torch.Tensor, bias, resid, gamma, beta, eps: float, dtype, resid_dtype,
+                  out_act=None, out_resid=None, stream=None):
+    """et_layernorm_fwd: LN(sum(part) + bias + resid)."""
+    nparts, M, N = part.shape
+    _check(_ln(part.data_ptr(), nparts, M, N, _ptr(bias), dtype_code(dtype), _ptr(resid), dtype_code(resid_dtype),
+               gamma.data_ptr(), beta.data_ptr(), eps, _ptr(out_act), _ptr(out_resid), _stream(stream)))
+    return out_act, out_resid
+
+
+def attn_short_max(d_k: int) -> int:
+    return int(_short_max(d_k))

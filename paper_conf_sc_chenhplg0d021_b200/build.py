@@ -1,0 +1,84 @@
+"""Build libet.so (the C-ABI library) in-tree for sm_100a.
+
+    python -m paper_conf_sc_chenhplg0d021_b200.build      (or __graft_entry__.build())
+
+Every .cu under csrc/ is compiled with
+    nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -lineinfo -Xcompiler -fPIC
+(NOT -arch=sm_100a: that emits compute_100 PTX and ptxas rejects tcgen05) and linked into
+paper_conf_sc_chenhplg0d021_b200/libet.so with the static CUDA runtime.  Objects are cached
+by source/header mtime in build/.
+"""
+from __future__ import annotations
+
+import concurrent.futures as cf
+import glob
+import os
+import shutil
+import subprocess
+import sys
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(PKG)
+CSRC = os.path.join(PKG, "csrc")
+INCLUDE = os.path.join(ROOT, "include")
+BUILD = os.path.join(ROOT, "build", "et")
+LIB = os.path.join(PKG, "libet.so")
+
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
+         "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC]
+
+
+def _nvcc() -> str:
+    for cand in (os.environ.get("NVCC"), shutil.which("nvcc"), "/usr/local/cuda/bin/nvcc"):
+        if cand and os.path.exists(cand):
+            return cand
+    raise RuntimeError("nvcc not found")
+
+
+def _headers() -> list[str]:
+    return glob.glob(os.path.join(CSRC, "**", "*.cuh"), recursive=True) + \
+        glob.glob(os.path.join(CSRC, "**", "*.h"), recursive=True) + \
+        glob.glob(os.path.join(INCLUDE, "*.h"))
+
+
+def sources() -> list[str]:
+    return sorted(glob.glob(os.path.join(CSRC, "**", "*.cu"), recursive=True))
+
+
+def build(verbose: bool = False, force: bool = False, debug: bool = False) -> str:
+    """Compile every .cu and link libet.so (debug=True: -DET_WATCHDOG build into build/et_dbg/libet_dbg.so)."""
+    nvcc = _nvcc()
+    bdir = BUILD + ("_dbg" if debug else "")
+    lib = os.path.join(bdir, "libet_dbg.so") if debug else LIB
+    flags = FLAGS + (["-DET_WATCHDOG"] if debug else [])
+    os.makedirs(bdir, exist_ok=True)
+    hdr_mtime = max([os.path.getmtime(h) for h in _headers()] + [0.0])
+    jobs = []
+    objs = []
+    for src in sources():
+        rel = os.path.relpath(src, CSRC).replace(os.sep, "_")
+        obj = os.path.join(bdir, rel + ".o")
+        objs.append(obj)
+        if force or not os.path.exists(obj) or os.path.getmtime(obj) < max(os.path.getmtime(src), hdr_mtime):
+            jobs.append([nvcc, *ARCH, *flags, "-c", src, "-o", obj])
+
+    def run(cmd):
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError("compile failed:\n" + " ".join(cmd) + "\n" + r.stdout + r.stderr)
+        if verbose and (r.stdout or r.stderr):
+            print(r.stdout + r.stderr, file=sys.stderr)
+
+    with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
+        list(ex.map(run, jobs))
+    if jobs or force or not os.path.exists(lib) or os.path.getmtime(lib) < max(os.path.getmtime(o) for o in objs):
+        tmp = lib + ".tmp"
+        run([nvcc, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-ldl",
+             "-lrt", "-lpthread"])
+        os.replace(tmp, lib)
+    return lib
+
+
+if __name__ == "__main__":
+    print(build(verbose=True, force="--force" in sys.argv, debug="--debug" in sys.argv))

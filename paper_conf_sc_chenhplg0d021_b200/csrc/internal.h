@@ -1,0 +1,111 @@
+// Internal host-side declarations shared by the C-ABI implementation (api.cu) and the kernel
+// launch wrappers (kernels/*.cu).  Not part of the public ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdarg>
+#include <cstdint>
+#include <cstddef>
+
+#include "et.h"
+
+namespace et {
+
+// thread-local error message (et_last_error)
+void set_error(const char* fmt, ...);
+et_status fail(et_status s, const char* fmt, ...);
+
+#define ET_TRY(expr)                 \
+  do {                               \
+    et_status _s = (expr);           \
+    if (_s != ET_OK) return _s;      \
+  } while (0)
+
+#define ET_CUDA(expr)                                                                              \
+  do {                                                                                             \
+    cudaError_t _e = (expr);                                                                       \
+    if (_e != cudaSuccess)                                                                         \
+      return ::et::fail(ET_ERR_CUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(_e), __FILE__, \
+                        __LINE__);                                                                 \
+  } while (0)
+
+inline size_t dtype_size(et_dtype d) { return d == ET_FP32 ? 4 : 2; }
+inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+inline bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+// ---------------------------------------------------------------- prune / pack (kernels/prune_pack.cu)
+struct PruneArgs {
+  const void* W;
+  int rows, cols;
+  et_dtype dtype;
+  et_pattern pattern;
+  int tile_r, tile_c, group_rows;
+  int n_prune;
+  const uint32_t* mask_in;
+};
+size_t prune_workspace_bytes(int rows, int cols, et_pattern pattern, int tile_r, int tile_c);
+// Runs the whole pack on `stream`; writes counts (nnz, rows_padded) to host via a sync.
+et_status prune_pack_run(const PruneArgs& a, et_packed_weight* out, void* ws, size_t ws_bytes, cudaStream_t stream);
+et_status unpack_run(const et_packed_weight* w, void* dense, cudaStream_t stream);
+
+// ---------------------------------------------------------------- tile-sparse GEMM (kernels/tsgemm.cu)
+// A segment of output tile-rows backed by one packed weight (QKV fuses three segments).
+struct GemmSegment {
+  const int32_t* row_ptr;   // tile CSR of the packed weight
+  const int32_t* tile_col;  // tile column per packed tile
+  const void* values;       // packed tiles
+  const void* bias;         // [seg_rows] in dtype, or nullptr
+  int tile_rows;            // number of 16-row tile rows in this segment
+  int out_col;              // first output column of the segment in Y
+  float scale;              // epilogue scale for ET_EPI_BIAS_SCALE (applied if apply_scale)
+  int apply_scale;
+};
+struct GemmArgs {
+  const void* X;            // [M, ldx] in dtype; columns [k0, k0 + K) are the GEMM's K range
+  int M, K, ldx, k0;
+  et_dtype dtype;
+  GemmSegment seg[3];
+  int nseg;
+  int kpart_tiles;          // split-K: number of 16-wide K tiles per part (K/16 = no split)
+  void* Y;                  // output [M, ldy] (dtype) or fp32 partials [nparts][M, ldy]
+  int ldy;
+  et_epilogue epi;
+};
+et_status gemm_run(const GemmArgs& a, cudaStream_t stream);
+
+// ---------------------------------------------------------------- LayerNorm (kernels/layernorm.cu)
+struct LnArgs {
+  const float* part;
+  int nparts, M, N;
+  const void* bias;
+  et_dtype dtype;
+  const void* resid;
+  et_dtype resid_dtype;
+  const float* gamma;
+  const float* beta;
+  float eps;
+  void* out_act;
+  void* out_resid;
+};
+et_status layernorm_run(const LnArgs& a, cudaStream_t stream);
+
+// ---------------------------------------------------------------- attention (kernels/attention.cu)
+struct AttnArgs {
+  const void* qkv;
+  int ld_qkv, q_off, k_off, v_off;
+  const int32_t* v_col;     // [H] or nullptr
+  const int32_t* v_width;   // [H] or nullptr
+  void* Z;
+  int ld_z;
+  const int32_t* z_col;     // [H] or nullptr
+  const int32_t* lengths;   // [B] or nullptr
+  int batch, seq_len, heads, d_k, head_begin, head_end;
+  int causal;
+  int long_form;
+  int v_width_max;          // upper bound of the per-head V width (multiple of 16)
+  float scale;
+  et_dtype dtype;
+};
+et_status attention_run(const AttnArgs& a, cudaStream_t stream);
+int attn_short_max(int d_k);
+
+}  // namespace et

@@ -1,0 +1,428 @@
+// Tile-sparse linear layer on tcgen05 (§4.2: tensor-tile pruning keeps or
+// drops whole 16x16 tiles; line 252: tile-pruned linear vs dense GEMM).
+//
+//   Y[m, n] = epilogue( sum over KEPT tiles (i, j) of X[m, 16j:16j+16] . W'[16i:16i+16, 16j:16j+16]^T )
+//
+// One tcgen05.mma (M=128 tokens, N=16 features, K=16) per kept tile; pruned tiles cost nothing.
+// Design (measured in profiles/r01/M1_tcgen05_probe.md):
+//   * the activation block (128 tokens x K<=768) lives in TMEM as the MMA A operand ("TS" MMA):
+//     TMA (SWIZZLE_128B) -> shared memory -> tcgen05.cp.  With A in shared memory every N=16 MMA
+//     re-reads 4 KB of A and the kernel is capped near 20 % of peak by smem bandwidth.
+//   * packed tiles (512 B each, core-matrix layout) are contiguous per (K part, tile row) and are
+//     streamed with 1-D bulk copies through an 8-stage shared-memory ring.
+//   * 8 MMA warps, one accumulator (16 TMEM columns) each, so 8 independent accumulation chains are
+//     in flight (one warp can only issue an MMA every ~60 cycles; a chain step takes ~110).
+//     Warps 0-3 and 4-7 form two warpgroups working on alternate "quads" of 4 tile rows; a
+//     warpgroup drains its 4 accumulators (tcgen05.ld) while the other one issues MMAs.
+//   * warp 8 fills A (TMA + tcgen05.cp), warp 9 streams the tiles and owns the TMEM allocation.
+// Grid: x = piece (a tile-row range of one segment), y = 128-token block, z = K part (split-K,
+// fp32 partial outputs, reduced by the LayerNorm kernel).
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cuda_fp16.h>
+#include <cuda_bf16.h>
+#include <cstdint>
+#include <mutex>
+#include <type_traits>
+
+#include "../internal.h"
+#include "../ptx.cuh"
+
+namespace et {
+namespace {
+
+constexpr int kMaxPieces = 64;
+constexpr int kNXS = 4;          // X staging stages (16 KB each: 128 rows x 64 K)
+constexpr int kNBS = 8;          // tile staging stages
+constexpr int kChunkTiles = 32;  // tiles per stage (16 KB)
+constexpr int kMaxKChunks = 12;  // K <= 768 per part
+constexpr int kMaxBChunks = 192; // tile chunks per CTA (one single-use full barrier each)
+constexpr int kAccCol = 384;     // first accumulator column (A uses [0, Kp/2) <= 384)
+constexpr int kThreads = 320;
+
+struct SegDev {
+  const int32_t* prp;       // part_row_ptr [kparts][tile_rows + 1]
+  const int32_t* tile_col;  // values order
+  const uint8_t* values;
+  const void* bias;
+  int tile_rows;
+  int out_col;
+  float scale;
+  int apply_scale;
+};
+struct Piece {
+  int16_t seg;
+  int16_t i0, i1;  // tile rows [i0, i1) of the segment
+};
+struct Params {
+  int M, Kp, kparts;
+  int nseg;
+  SegDev seg[3];
+  int npieces;
+  Piece piece[kMaxPieces];
+  void* Y;
+  int ldy;
+  long long part_stride;   // elements between split-K partial outputs (fp32 epilogue)
+};
+
+struct __align__(8) Barriers {
+  uint64_t xfull[kNXS], xempty[kNXS], afill[kMaxKChunks], accf[8], bfull[kMaxBChunks];
+  uint32_t tmem_base;
+  int quads_done[2];   // per warpgroup, written by its leader thread after each quad
+};
+
+constexpr size_t kSmemX = (size_t)kNXS * 16384;
+constexpr size_t kSmemB = (size_t)kNBS * kChunkTiles * 512;
+constexpr size_t kSmemBytes = 1024 + kSmemX + kSmemB + sizeof(Barriers);
+
+__device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * (1.0f + erff(x * 0.70710678118654752f)); }
+
+template <int kEpi, bool kBF16>
+__device__ __forceinline__ void epilogue_store(const Params& p, const SegDev& sg, int row_g, int col_local,
+                                               const float (&acc)[16], int z) {
+  // col_local: first output feature of this 16-wide group within the segment
+  using T = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
+  if constexpr (kEpi == ET_EPI_F32) {
+    float* Y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row_g * p.ldy + sg.out_col + col_local;
+#pragma unroll
+    for (int c = 0; c < 16; c += 4)
+      *reinterpret_cast<float4*>(Y + c) = make_float4(acc[c], acc[c + 1], acc[c + 2], acc[c + 3]);
+  } else {
+    float v[16];
+    const T* b = static_cast<const T*>(sg.bias);
+#pragma unroll
+    for (int c = 0; c < 16; ++c) {
+      float x = acc[c];
+      if (b) {
+        if constexpr (kBF16) x += __bfloat162float(b[col_local + c]);
+        else x += __half2float(b[col_local + c]);
+      }
+      if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
+        if (sg.apply_scale) x *= sg.scale;
+      } else if constexpr (kEpi == ET_EPI_BIAS_GELU) {
+        x = gelu_erf(x);
+      } else if constexpr (kEpi == ET_EPI_BIAS_RELU) {
+        x = fmaxf(x, 0.0f);
+      }
+      v[c] = x;
+    }
+    uint32_t packed[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) packed[c] = pack2<kBF16>(v[2 * c], v[2 * c + 1]);
+    T* Y = static_cast<T*>(p.Y) + (size_t)row_g * p.ldy + sg.out_col + col_local;
+    *reinterpret_cast<uint4*>(Y) = make_uint4(packed[0], packed[1], packed[2], packed[3]);
+    *reinterpret_cast<uint4*>(Y + 8) = make_uint4(packed[4], packed[5], packed[6], packed[7]);
+  }
+}
+
+template <int kEpi, bool kBF16>
+__global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
+                                                             const __grid_constant__ Params p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sX = smem;
+  uint8_t* sB = smem + kSmemX;
+  Barriers& bar = *reinterpret_cast<Barriers*>(smem + kSmemX + kSmemB);
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const Piece pc = p.piece[blockIdx.x];
+  const SegDev& sg = p.seg[pc.seg];
+  const int m0 = blockIdx.y * 128;
+  const int z = blockIdx.z;
+  const int nk = p.Kp / 64;                    // A chunks (64 K each)
+  const int32_t* rp = sg.prp + (size_t)z * (sg.tile_rows + 1);
+  const int pb = rp[pc.i0], pe = rp[pc.i1];    // this CTA's packed tiles [pb, pe)
+  const int nchunks = (pe - pb + kChunkTiles - 1) / kChunkTiles;
+  const int nrows = pc.i1 - pc.i0;
+  const int nquads = (nrows + 3) / 4;
+
+  if (nchunks > kMaxBChunks) __trap();   // host sizes pieces so this cannot happen
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kNXS; ++i) {
+      mbar_init(&bar.xfull[i], 1);
+      mbar_init(&bar.xempty[i], 1);
+    }
+    for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.afill[i], 1);
+    // one full barrier per tile chunk, each completing exactly once (parity 0): a warp may skip
+    // ahead to a chunk whose ring slot has not even received its previous fill, and a parity wait
+    // on a reused barrier cannot tell those phases apart.
+    for (int i = 0; i < nchunks; ++i) mbar_init(&bar.bfull[i], 1);
+    bar.quads_done[0] = bar.quads_done[1] = 0;
+    for (int i = 0; i < 8; ++i) mbar_init(&bar.accf[i], 1);
+    fence_mbar_init();
+  }
+  if (warp == 9) tmem_alloc<512>(&bar.tmem_base);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = bar.tmem_base;
+
+  if (warp == 8) {
+    // ===================== A producer: X block -> smem (TMA) -> TMEM (tcgen05.cp)
+    if (lane == 0) {
+      tma_prefetch_desc(&tmap_x);
+      const int kx0 = z * p.Kp;
+      for (int j = 0; j < nk && j < kNXS; ++j) {
+        mbar_expect_tx(&bar.xfull[j], 16384);
+        tma_load_2d(sX + j * 16384, &tmap_x, &bar.xfull[j], kx0 + j * 64, m0);
+      }
+      for (int j = 0; j < nk; ++j) {
+        const int slot = j % kNXS;
+        mbar_wait(&bar.xfull[slot], (j / kNXS) & 1);
+        tc_fence_after();
+        const uint32_t src = smem_u32(sX + slot * 16384);
+#pragma unroll
+        for (int s = 0; s < 4; ++s)
+          tmem_cp_128x256b(tbase + j * 32 + s * 8, make_sdesc(src + s * 32, 16, 1024, kLayoutSW128));
+        mma_commit(&bar.afill[j]);
+        mma_commit(&bar.xempty[slot]);
+        // refill the slot of the PREVIOUS chunk (its copy has had time to finish) with chunk j-1+NXS
+        const int jr = j - 1;
+        if (jr >= 0 && jr + kNXS < nk) {
+          const int rs = jr % kNXS;
+          mbar_wait(&bar.xempty[rs], (jr / kNXS) & 1);
+          mbar_expect_tx(&bar.xfull[rs], 16384);
+          tma_load_2d(sX + rs * 16384, &tmap_x, &bar.xfull[rs], kx0 + (jr + kNXS) * 64, m0);
+        }
+      }
+    }
+  } else if (warp == 9) {
+    // ===================== tile producer: packed tiles -> smem ring (bulk copies)
+    // Slot reuse is quad-granular: chunk c may overwrite chunk c - kNBS once every quad (4 tile
+    // rows) touching chunk c - kNBS has completed its MMAs.  Warpgroup g owns quads g, g+2, ...
+    // and bumps quads_done[g] after each quad's epilogue barrier (its MMAs are complete then).
+    if (lane == 0) {
+      const uint8_t* vals = sg.values + (size_t)pb * 512;
+      int qq = 0;             // last quad that starts before the end of the chunk being recycled
+      for (int c = 0; c < nchunks; ++c) {
+        const int slot = c % kNBS;
+        if (c >= kNBS) {
+          const int cr = c - kNBS;
+          const int end_tile = pb + (cr + 1) * kChunkTiles;   // tiles of chunk cr are < end_tile
+          while (qq + 1 < nquads && rp[min(pc.i0 + (qq + 1) * 4, pc.i1)] < end_tile) ++qq;
+          const int need0 = qq / 2 + 1, need1 = (qq + 1) / 2;   // quads 0,2,.. / 1,3,.. up to qq
+          while (ld_acquire_shared(&bar.quads_done[0]) < need0) {}
+          while (ld_acquire_shared(&bar.quads_done[1]) < need1) {}
+        }
+        const int nt = min(kChunkTiles, pe - pb - c * kChunkTiles);
+        mbar_expect_tx(&bar.bfull[c], nt * 512);
+        bulk_load(sB + slot * (kChunkTiles * 512), vals + (size_t)c * kChunkTiles * 512, nt * 512, &bar.bfull[c]);
+      }
+    }
+  } else {
+    // ===================== MMA + epilogue warps (2 warpgroups x 4 warps)
+    const int g = warp >> 2, jw = warp & 3;
+    const uint32_t idesc = make_idesc_f16(128, 16, kBF16 ? 1 : 0, 0, 0);
+    const uint32_t d_tmem = tbase + kAccCol + warp * 16;
+    const uint32_t sB_u32 = smem_u32(sB);
+    const int kbase = z * 48;   // first tile column of this K part
+    int a_ready = -1;           // highest A chunk known filled
+    int cur_chunk = -1;         // B chunk whose full barrier was last waited
+    int round = 0;
+    for (int q = g; q < nquads; q += 2, ++round) {
+      const int t = q * 4 + jw;                 // local tile row of this warp in this round
+      if (t < nrows) {
+        const int i = pc.i0 + t;
+        const int p0 = rp[i], p1 = rp[i + 1];
+        for (int base = p0; base < p1; base += 32) {
+          const int mycol = (base + lane < p1) ? sg.tile_col[base + lane] : 0;
+          const int n = min(32, p1 - base);
+          for (int u = 0; u < n; ++u) {
+            const int pp = base + u;
+            const int kc = __shfl_sync(0xffffffffu, mycol, u) - kbase;
+            const int c = (pp - pb) / kChunkTiles;
+            if (c != cur_chunk) {
+              mbar_wait_warp(&bar.bfull[c], 0);
+              cur_chunk = c;
+              tc_fence_after();
+            }
+            const int ach = kc >> 2;
+            if (ach > a_ready) {
+              mbar_wait_warp(&bar.afill[ach], 0);
+              a_ready = ach;
+              tc_fence_after();
+            }
+            const uint32_t baddr = sB_u32 + (c % kNBS) * (kChunkTiles * 512) + ((pp - pb) % kChunkTiles) * 512;
+            mma_ts_warp(d_tmem, tbase + kc * 8, make_sdesc(baddr, 128, 256, kLayoutNone), idesc, pp != p0);
+          }
+        }
+      }
+      mma_commit_warp(&bar.accf[warp]);
+
+      // ---- epilogue of quad q: this warp reads lane quarter jw of the 4 accumulators of its group
+      float acc[4][16];
+#pragma unroll
+      for (int a = 0; a < 4; ++a) mbar_wait_warp(&bar.accf[g * 4 + a], round & 1);
+      tc_fence_after();
+#pragma unroll
+      for (int a = 0; a < 4; ++a) {
+        uint32_t r[16];
+        tmem_ld16(tbase + kAccCol + (g * 4 + a) * 16 + ((uint32_t)(jw * 32) << 16), r);
+        tmem_ld_wait();
+#pragma unroll
+        for (int c = 0; c < 16; ++c) acc[a][c] = __uint_as_float(r[c]);
+      }
+      tc_fence_before();
+      named_bar_sync(1 + g, 128);
+      __syncwarp();
+      if (jw == 0 && lane == 0) st_release_shared(&bar.quads_done[g], round + 1);   // quad's MMAs complete
+      const int row_g = m0 + jw * 32 + lane;
+#pragma unroll
+      for (int a = 0; a < 4; ++a) {
+        const int ta = q * 4 + a;
+        if (ta >= nrows) continue;
+        const int i = pc.i0 + ta;
+        if (rp[i + 1] == rp[i]) {   // fully pruned tile row: the accumulator was never written
+#pragma unroll
+          for (int c = 0; c < 16; ++c) acc[a][c] = 0.0f;
+        }
+        if (row_g < p.M) epilogue_store<kEpi, kBF16>(p, sg, row_g, i * 16, acc[a], z);
+      }
+    }
+  }
+
+  __syncwarp();   // producer warps: lane 0 ran the loops alone; reconverge before the block barrier
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 9) {
+    __syncwarp();
+    tc_fence_after();
+    tmem_dealloc<512>(tbase);   // .sync.aligned: the whole warp, converged
+  }
+}
+
+// ---------------------------------------------------------------- host side
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode() {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(ptr);
+  });
+  return fn;
+}
+
+template <int kEpi, bool kBF16>
+et_status launch_typed(const CUtensorMap& tm, const Params& prm, dim3 grid, cudaStream_t stream) {
+  auto kern = tsgemm_kernel<kEpi, kBF16>;
+  static std::once_flag once;
+  static cudaError_t attr_err = cudaSuccess;
+  std::call_once(once, [&] {
+    attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  });
+  ET_CUDA(attr_err);
+  kern<<<grid, kThreads, kSmemBytes, stream>>>(tm, prm);
+  ET_CUDA(cudaGetLastError());
+  return ET_OK;
+}
+
+}  // namespace
+
+et_status make_tmap_2d(CUtensorMap* tm, const void* base, et_dtype dtype, uint64_t rows, uint64_t cols,
+                       uint64_t ld_elems, uint32_t box_cols, uint32_t box_rows, bool swizzle128) {
+  EncodeTiledFn enc = get_encode();
+  if (!enc) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {ld_elems * dtype_size(dtype)};
+  cuuint32_t box[2] = {box_cols, box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUtensorMapDataType dt = dtype == ET_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                           : dtype == ET_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                              : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
+  CUresult r = enc(tm, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return ET_OK;
+}
+
+et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
+  if (a.dtype == ET_FP32) return fail(ET_ERR_UNSUPPORTED, "tile GEMM: FP32 operands not implemented in this build");
+  if (a.K % 64) return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K must be a multiple of 64 (got %d)", a.K);
+  if (!aligned16(a.X) || (a.ldx * 2) % 16 || (a.k0 * 2) % 16)
+    return fail(ET_ERR_INVALID_ARG, "tile GEMM: X must be 16-byte aligned with 16-byte row pitch");
+  const int kparts = (a.K + 767) / 768;
+  if (kparts > 1 && a.epi != ET_EPI_F32)
+    return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K > 768 needs the fp32 split-K epilogue");
+  if (a.K % kparts || (a.K / kparts) % 64 || a.K / kparts > 768 || (kparts > 1 && a.K / kparts != 768 && a.K != kparts * 768))
+    return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K=%d not splittable into parts of 768", a.K);
+  if (a.M <= 0) return ET_OK;
+
+  Params prm{};
+  prm.M = a.M;
+  prm.Kp = kparts > 1 ? 768 : a.K;
+  prm.kparts = kparts;
+  prm.nseg = a.nseg;
+  prm.Y = a.Y;
+  prm.ldy = a.ldy;
+  prm.part_stride = (long long)a.M * a.ldy;
+  const int mblocks = (a.M + 127) / 128;
+  int total_rows = 0;
+  for (int s = 0; s < a.nseg; ++s) total_rows += a.seg[s].tile_rows;
+  // pieces: aim for ~1-2 waves of CTAs over 148 SMs, >= 8 tile rows per piece
+  const int target_ctas = 148;
+  int pieces_total = (target_ctas + mblocks * kparts - 1) / (mblocks * kparts);
+  if (pieces_total < a.nseg) pieces_total = a.nseg;
+  int np = 0;
+  for (int s = 0; s < a.nseg; ++s) {
+    const GemmSegment& gs = a.seg[s];
+    prm.seg[s].prp = gs.row_ptr;
+    prm.seg[s].tile_col = gs.tile_col;
+    prm.seg[s].values = static_cast<const uint8_t*>(gs.values);
+    prm.seg[s].bias = gs.bias;
+    prm.seg[s].tile_rows = gs.tile_rows;
+    prm.seg[s].out_col = gs.out_col;
+    prm.seg[s].scale = gs.scale;
+    prm.seg[s].apply_scale = gs.apply_scale;
+    int ps = (int)(((long long)pieces_total * gs.tile_rows * 2 + (total_rows > 0 ? total_rows : 1)) /
+                   (2LL * (total_rows > 0 ? total_rows : 1)));   // rounded
+    if (ps < 1) ps = 1;
+    if (ps > gs.tile_rows / 8) ps = gs.tile_rows / 8 > 0 ? gs.tile_rows / 8 : 1;
+    // each piece's tile stream must fit kMaxBChunks chunks
+    for (;;) {
+      bool ok = true;
+      for (int k = 0; k < ps && ok; ++k) {
+        const int i0 = (int)((long long)gs.tile_rows * k / ps), i1 = (int)((long long)gs.tile_rows * (k + 1) / ps);
+        ok = (long long)(i1 - i0) * (a.K / 16) <= (long long)kMaxBChunks * kChunkTiles;
+      }
+      if (ok || ps >= gs.tile_rows) break;
+      ++ps;
+    }
+    for (int k = 0; k < ps; ++k) {
+      if (np >= kMaxPieces) return fail(ET_ERR_INTERNAL, "tile GEMM: too many pieces");
+      prm.piece[np].seg = (int16_t)s;
+      prm.piece[np].i0 = (int16_t)((long long)gs.tile_rows * k / ps);
+      prm.piece[np].i1 = (int16_t)((long long)gs.tile_rows * (k + 1) / ps);
+      ++np;
+    }
+  }
+  prm.npieces = np;
+  CUtensorMap tm;   // the K offset k0 is folded into the base address
+  ET_TRY(make_tmap_2d(&tm, static_cast<const uint8_t*>(a.X) + (size_t)a.k0 * 2, a.dtype, (uint64_t)a.M,
+                      (uint64_t)a.K, (uint64_t)a.ldx, 64, 128, true));
+  dim3 grid(np, mblocks, kparts);
+  const bool bf = a.dtype == ET_BF16;
+  switch (a.epi) {
+    case ET_EPI_BIAS: return bf ? launch_typed<ET_EPI_BIAS, true>(tm, prm, grid, stream)
+                                : launch_typed<ET_EPI_BIAS, false>(tm, prm, grid, stream);
+    case ET_EPI_BIAS_SCALE: return bf ? launch_typed<ET_EPI_BIAS_SCALE, true>(tm, prm, grid, stream)
+                                      : launch_typed<ET_EPI_BIAS_SCALE, false>(tm, prm, grid, stream);
+    case ET_EPI_BIAS_GELU: return bf ? launch_typed<ET_EPI_BIAS_GELU, true>(tm, prm, grid, stream)
+                                     : launch_typed<ET_EPI_BIAS_GELU, false>(tm, prm, grid, stream);
+    case ET_EPI_BIAS_RELU: return bf ? launch_typed<ET_EPI_BIAS_RELU, true>(tm, prm, grid, stream)
+                                     : launch_typed<ET_EPI_BIAS_RELU, false>(tm, prm, grid, stream);
+    case ET_EPI_F32: return bf ? launch_typed<ET_EPI_F32, true>(tm, prm, grid, stream)
+                               : launch_typed<ET_EPI_F32, false>(tm, prm, grid, stream);
+  }
+  return fail(ET_ERR_INVALID_ARG, "tile GEMM: bad epilogue %d", (int)a.epi);
+}
+
+}  // namespace et
