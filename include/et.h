@@ -178,16 +178,18 @@ typedef struct {
 int32_t et_attn_short_max(int32_t d_k);
 
 /* Attention core (steps 2-6 of Fig. 3(a)):
- *   Z[:, h*dv : (h+1)*dv] = softmax(mask(Q_h . K_h^T * scale)) . V_h      for h in [head_begin, head_end)
- * qkv: [batch*seq_len, ld_qkv] holding Q at column q_off + h*d_k, K at k_off + h*d_k and V at
- * v_off + v_col[h] (v_col / v_width: device int32 [heads] or NULL for V laid out like Q, i.e.
- * v_col[h] = h*d_k, v_width[h] = d_k).  `scale` multiplies the scores (pass 1 if Q was already
- * scaled by 1/sqrt(d_k), the reordered form of line 159).  Z: [batch*seq_len, ld_z], head h
- * written at column z_col[h] (NULL => h*d_k) — V widths padded to 16 with zero rows write
- * zeros.  The seq x seq score matrix never leaves TMEM / registers. */
+ *   Z_h = softmax(mask(Q_h . K_h^T * scale)) . V_h      for h in [head_begin, head_end)
+ * qkv: [batch*seq_len, ld_qkv] (16-byte aligned rows) holding Q_h at column q_off + h*d_k and K_h at
+ * k_off + h*d_k.  V_h starts at column v_off + v_col[h] and is v_width[h] wide (device int32 [H];
+ * NULL => v_col[h] = h*d_k, v_width[h] = d_k); v_width_max bounds v_width (multiple of 16, <= d_k).
+ * `scale` multiplies the scores: pass 1 when Q was already scaled by 1/sqrt(d_k) (the reordering
+ * of line 159, §3.3).  Z: [batch*seq_len, ld_z]; head h's column c goes to Z column h*d_k + c, or
+ * to z_map[v_col[h] + c] when z_map (device int32 over the packed V columns, -1 = skip) is given
+ * (row-pruned W_V, line 171).  Rows >= len_b of a sequence are computed like any other query.
+ * The seq x seq score matrix never leaves TMEM / registers. */
 et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld_qkv, int32_t q_off, int32_t k_off,
-                           int32_t v_off, const int32_t* v_col, const int32_t* v_width, float scale, void* Z,
-                           int32_t ld_z, const int32_t* z_col, void* stream);
+                           int32_t v_off, const int32_t* v_col, const int32_t* v_width, int32_t v_width_max,
+                           float scale, void* Z, int32_t ld_z, const int32_t* z_map, void* stream);
 
 /* Self-attention block (Fig. 3(a) steps 1-7, Eq. 3-4):
  *   out = SelfAttn(X)                  if ln_gamma == NULL

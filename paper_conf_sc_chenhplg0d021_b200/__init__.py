@@ -232,3 +232,137 @@ def layernorm_fwd(part: torch.Tensor, bias, resid, gamma, beta, eps: float, dtyp
 
 def attn_short_max(d_k: int) -> int:
     return int(_short_max(d_k))
+
+
+# ------------------------------------------------------------------------------------------ attention
+_core = _sig("et_attn_core_fwd", ctypes.c_int,
+             [ctypes.POINTER(AttnDescC), _vp, _i32, _i32, _i32, _i32, _vp, _vp, _i32, _f32, _vp, _i32, _vp, _vp])
+_attn_ws = _sig("et_attention_workspace_size", ctypes.c_int,
+                [ctypes.POINTER(AttnDescC), ctypes.POINTER(PackedWeightC), ctypes.POINTER(_sz)])
+_attn = _sig("et_attention_fwd", ctypes.c_int,
+             [ctypes.POINTER(AttnDescC), _vp] + [ctypes.POINTER(PackedWeightC)] * 4 + [_vp] * 6 +
+             [_f32, _vp, _vp, _sz, _vp])
+_enc_ws = _sig("et_encoder_workspace_size", ctypes.c_int,
+               [ctypes.POINTER(AttnDescC), _i32, _i32, ctypes.c_int, ctypes.POINTER(LayerC), ctypes.POINTER(_sz)])
+_enc = _sig("et_encoder_fwd", ctypes.c_int,
+            [ctypes.POINTER(AttnDescC), _i32, _i32, ctypes.c_int, _f32, ctypes.c_int, ctypes.POINTER(LayerC), _vp,
+             _vp, _vp, _sz, _vp])
+
+
+def attn_desc(batch, seq_len, heads, d_model, dtype, lengths=None, causal=False, mode="auto",
+              head_begin=0, head_end=None) -> AttnDescC:
+    d = AttnDescC()
+    d.batch, d.seq_len, d.heads, d.d_model = batch, seq_len, heads, d_model
+    d.dtype = dtype_code(dtype)
+    d.lengths_dev = _ptr(lengths)
+    d.causal = 1 if causal else 0
+    d.mode = _MODE[mode] if isinstance(mode, str) else mode
+    d.head_begin = head_begin
+    d.head_end = heads if head_end is None else head_end
+    return d
+
+
+def attn_core_fwd(qkv: torch.Tensor, batch: int, seq_len: int, heads: int, d_model: int, q_off: int, k_off: int,
+                  v_off: int, lengths=None, causal=False, mode="auto", scale: float = 1.0, v_col=None,
+                  v_width=None, v_width_max: int = 0, Z=None, z_map=None, stream=None):
+    """et_attn_core_fwd: on-the-fly attention on a [batch*seq_len, ld] QKV buffer."""
+    d = attn_desc(batch, seq_len, heads, d_model, qkv.dtype, lengths, causal, mode)
+    if Z is None:
+        Z = torch.zeros(batch * seq_len, d_model, dtype=qkv.dtype, device=qkv.device)
+    _check(_core(ctypes.byref(d), qkv.data_ptr(), qkv.stride(0), q_off, k_off, v_off, _ptr(v_col), _ptr(v_width),
+                 v_width_max, scale, Z.data_ptr(), Z.stride(0), _ptr(z_map), _stream(stream)))
+    return Z
+
+
+# ------------------------------------------------------------------------------------------ layers
+class Layer:
+    """One packed encoder layer: six packed weights + device biases / LayerNorm parameters."""
+
+    def __init__(self, packed: dict, dense: dict):
+        self.packed = packed      # name -> Packed
+        self.dense = dense        # biases (dtype) and LN params (fp32) as device tensors
+        c = LayerC()
+        for n in ("wq", "wk", "wv", "wo", "w1", "w2"):
+            setattr(c, n, packed[n].c)
+        for n in ("bq", "bk", "bv", "bo", "b1", "b2", "ln1_g", "ln1_b", "ln2_g", "ln2_b"):
+            setattr(c, n, dense[n].data_ptr())
+        self.c = c
+
+
+def pack_layer(raw: dict, scheme: str, ratio: float, heads: int, dtype="fp16", stream=None) -> Layer:
+    """Prune + pack the six matrices of one layer (pattern per scheme: PAPER.md line 107, 317).
+
+    raw: name -> float32 numpy/torch array holding storage-dtype values (et_synth.make_layer)."""
+    tdt = torch_dtype(dtype)
+    dev = torch.device("cuda")
+    packed, dense = {}, {}
+    d_model = raw["wq"].shape[0]
+    for n in ("wq", "wk", "wv", "wo", "w1", "w2"):
+        W = torch.as_tensor(raw[n]).to(dev).to(tdt).contiguous()
+        if scheme == "none":
+            pat, r = "tile", 0.0
+        elif scheme == "attention-aware" and n == "wv":
+            pat, r = "row", ratio
+        else:
+            pat, r = "tile", ratio
+        packed[n] = prune_pack(W, pat, r, (16, 16), group_rows=d_model // heads if pat == "row" else 0,
+                               stream=stream)
+    for n in ("bq", "bk", "bv", "bo", "b1", "b2"):
+        dense[n] = torch.as_tensor(raw[n]).to(dev).to(tdt).contiguous()
+    for n in ("ln1_g", "ln1_b", "ln2_g", "ln2_b"):
+        dense[n] = torch.as_tensor(raw[n]).to(dev).to(torch.float32).contiguous()
+    return Layer(packed, dense)
+
+
+def attention_fwd(X: torch.Tensor, layer: Layer, batch: int, seq_len: int, heads: int, lengths=None,
+                  causal=False, mode="auto", ln: bool = True, ln_eps: float = 1e-12, out=None, stream=None):
+    """et_attention_fwd: LN(X + SelfAttn(X)) (ln=True) or SelfAttn(X)."""
+    d_model = X.shape[1]
+    d = attn_desc(batch, seq_len, heads, d_model, X.dtype, lengths, causal, mode)
+    P, D = layer.packed, layer.dense
+    nb = _sz()
+    _check(_attn_ws(ctypes.byref(d), ctypes.byref(P["wv"].c), ctypes.byref(nb)))
+    ws = torch.empty(nb.value, dtype=torch.uint8, device=X.device)
+    if out is None:
+        out = torch.empty_like(X)
+    _check(_attn(ctypes.byref(d), X.data_ptr(), ctypes.byref(P["wq"].c), ctypes.byref(P["wk"].c),
+                 ctypes.byref(P["wv"].c), ctypes.byref(P["wo"].c), D["bq"].data_ptr(), D["bk"].data_ptr(),
+                 D["bv"].data_ptr(), D["bo"].data_ptr(), D["ln1_g"].data_ptr() if ln else None,
+                 D["ln1_b"].data_ptr() if ln else None, ln_eps, out.data_ptr(), ws.data_ptr(), ws.numel(),
+                 _stream(stream)))
+    return out
+
+
+class Encoder:
+    """A packed encoder stack bound to a fixed problem shape: owns the C layer array and workspace."""
+
+    def __init__(self, layers: list, batch: int, seq_len: int, heads: int, d_ff: int, act="gelu", ln_eps=1e-12,
+                 dtype="fp16", resid_dtype="fp16", causal=False, mode="auto", lengths=None):
+        self.layers = layers
+        self.arr = (LayerC * len(layers))(*[l.c for l in layers])
+        d_model = layers[0].packed["wq"].c.rows
+        self.d_model = d_model
+        self.desc = attn_desc(batch, seq_len, heads, d_model, dtype, lengths, causal, mode)
+        self.lengths = lengths
+        self.d_ff, self.act, self.eps = d_ff, _ACT[act], ln_eps
+        self.dtype, self.resid_dtype = dtype_code(dtype), dtype_code(resid_dtype)
+        nb = _sz()
+        _check(_enc_ws(ctypes.byref(self.desc), len(layers), d_ff, self.resid_dtype, self.arr, ctypes.byref(nb)))
+        self.ws = torch.empty(nb.value, dtype=torch.uint8, device="cuda")
+
+    def set_lengths(self, lengths):
+        self.lengths = lengths
+        self.desc.lengths_dev = _ptr(lengths)
+
+    def __call__(self, X: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+        """et_encoder_fwd: X, out [batch*seq_len, d_model] in resid_dtype."""
+        if out is None:
+            out = torch.empty_like(X)
+        _check(_enc(ctypes.byref(self.desc), len(self.layers), self.d_ff, self.act, self.eps, self.resid_dtype,
+                    self.arr, X.data_ptr(), out.data_ptr(), self.ws.data_ptr(), self.ws.numel(), _stream(stream)))
+        return out
+
+
+def encoder_fwd(X: torch.Tensor, layers: list, batch: int, seq_len: int, heads: int, d_ff: int, **kw):
+    """One-shot et_encoder_fwd (allocates the workspace; use Encoder for repeated calls)."""
+    return Encoder(layers, batch, seq_len, heads, d_ff, **kw)(X)

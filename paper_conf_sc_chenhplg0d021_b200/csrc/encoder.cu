@@ -1,0 +1,382 @@
+// Host orchestration of the attention block and of the encoder stack (C ABI in include/et.h).
+// Every step below is a launch of one of the library's kernels on the caller's stream:
+//   1. QKV tile-sparse GEMM (three segments: W_Q, W_K, W_V), Q columns scaled by 1/sqrt(d_k) in
+//      FP32 before rounding — the scale moved before Q.K^T (§3.3);
+//   2. on-the-fly attention (short or long form, line 97-147);
+//   3. output projection (tile-sparse GEMM, fp32 result) — Eq. 4;
+//   4. residual + LayerNorm (line 75);
+//   5. FFN1 + activation, 6. FFN2 (split-K fp32 partials), 7. residual + LayerNorm (line 75).
+// No host synchronisation; CUDA-graph capturable.
+#include <cuda_runtime.h>
+#include <cmath>
+#include <vector>
+
+#include "internal.h"
+
+namespace et {
+namespace {
+
+struct Carver {
+  uint8_t* base;
+  size_t off = 0;
+  void* take(size_t bytes) {
+    off = align_up(off, 256);
+    void* p = base ? base + off : nullptr;
+    off += bytes;
+    return p;
+  }
+};
+
+bool long_form_for(const et_attn_desc* d) {
+  const int dk = d->d_model / d->heads;
+  if (d->mode == ET_ATTN_LONG) return true;
+  if (d->mode == ET_ATTN_SHORT) return false;
+  return d->seq_len > attn_short_max(dk);
+}
+
+et_status check_desc(const et_attn_desc* d) {
+  if (!d) return fail(ET_ERR_INVALID_ARG, "null attention descriptor");
+  if (d->batch <= 0 || d->seq_len <= 0 || d->heads <= 0 || d->d_model <= 0)
+    return fail(ET_ERR_INVALID_ARG, "batch, seq_len, heads, d_model must be positive");
+  if (d->d_model % d->heads) return fail(ET_ERR_INVALID_ARG, "d_model %% heads != 0");
+  if (d->dtype != ET_FP16 && d->dtype != ET_BF16)
+    return fail(ET_ERR_UNSUPPORTED, "forward path: dtype must be FP16 or BF16 in this build");
+  const int dk = d->d_model / d->heads;
+  if (dk != 64 && dk != 128) return fail(ET_ERR_UNSUPPORTED, "d_k must be 64 or 128 (got %d)", dk);
+  if (d->d_model % 64) return fail(ET_ERR_UNSUPPORTED, "d_model must be a multiple of 64");
+  if (d->mode == ET_ATTN_SHORT && d->seq_len > attn_short_max(dk))
+    return fail(ET_ERR_UNSUPPORTED, "short attention form needs seq_len <= %d", attn_short_max(dk));
+  if (d->head_begin < 0 || d->head_end > d->heads || d->head_begin >= d->head_end)
+    return fail(ET_ERR_INVALID_ARG, "bad head range [%d, %d)", d->head_begin, d->head_end);
+  return ET_OK;
+}
+
+et_status check_weight(const et_packed_weight* w, int rows, int cols, et_dtype dt, const char* name, bool allow_row) {
+  if (!w || !w->values) return fail(ET_ERR_INVALID_ARG, "%s: packed weight without values", name);
+  if (w->rows != rows || w->cols != cols)
+    return fail(ET_ERR_INVALID_ARG, "%s: shape %dx%d, expected %dx%d", name, w->rows, w->cols, rows, cols);
+  if (w->dtype != dt) return fail(ET_ERR_INVALID_ARG, "%s: dtype mismatch", name);
+  if (w->pattern == ET_PRUNE_ROW && !allow_row) return fail(ET_ERR_UNSUPPORTED, "%s: row pruning only for W_V", name);
+  if (w->pattern != ET_PRUNE_TILE && w->pattern != ET_PRUNE_ROW)
+    return fail(ET_ERR_UNSUPPORTED, "%s: pattern %d not supported by the forward path", name, (int)w->pattern);
+  return ET_OK;
+}
+
+GemmSegment seg_of(const et_packed_weight* w, const void* bias, int out_col) {
+  GemmSegment s{};
+  s.row_ptr = w->part_row_ptr;
+  s.tile_col = w->tile_col;
+  s.values = w->values;
+  s.bias = bias;
+  s.tile_rows = (w->pattern == ET_PRUNE_TILE ? w->rows : w->rows_padded) / 16;
+  s.out_col = out_col;
+  s.scale = 1.f;
+  s.apply_scale = 0;
+  return s;
+}
+
+// Workspace of one attention block (shared by the encoder).
+struct BlockWs {
+  void* qkv;        // [M, ldq]
+  int ldq;
+  void* z;          // [M, d]
+  float* part;      // [kparts_max][M, d]
+  int32_t* v_col;   // [H]   (attention-aware only)
+  int32_t* v_width; // [H]
+  void* bv_packed;  // [vmax]
+  void* bo_folded;  // [d]
+};
+
+int v_cols_of(const et_packed_weight* wv, int d) {
+  return wv->pattern == ET_PRUNE_ROW ? (int)align_up((size_t)std::max(wv->rows_padded, 16), 8) : d;
+}
+
+void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, BlockWs* ws) {
+  const size_t M = (size_t)d->batch * d->seq_len;
+  const size_t es = dtype_size(d->dtype);
+  ws->ldq = 2 * d->d_model + vmax;
+  ws->qkv = c.take(M * ws->ldq * es);
+  ws->z = c.take(M * d->d_model * es);
+  ws->part = static_cast<float*>(c.take((size_t)kparts_max * M * d->d_model * 4));
+  ws->v_col = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
+  ws->v_width = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
+  ws->bv_packed = c.take((size_t)vmax * es);
+  ws->bo_folded = c.take((size_t)d->d_model * es);
+}
+
+// Steps 1-3 (+4 when gamma != NULL): attention block on X (act dtype), output either the fp32
+// O-projection partial in ws->part (for the caller's LayerNorm) or written through `ln`.
+et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et_packed_weight* wq,
+                              const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
+                              const void* bq, const void* bk, const void* bv, const void* bo, const BlockWs& ws,
+                              const void** bo_eff, cudaStream_t st) {
+  const int dm = d->d_model, H = d->heads, dk = dm / H;
+  const int M = d->batch * d->seq_len;
+  const bool rowv = wv->pattern == ET_PRUNE_ROW;
+  const void* bv_use = bv;
+  *bo_eff = bo;
+  if (rowv) {
+    VPrep vp{wv, wo, bv, bo, H, dk, d->dtype, ws.v_col, ws.v_width, ws.bv_packed, ws.bo_folded};
+    ET_TRY(vprep_run(vp, st));
+    bv_use = ws.bv_packed;
+    *bo_eff = ws.bo_folded;
+    // pruned V features leave zero columns in Z (their constant b_V is folded into b_O')
+    ET_CUDA(cudaMemsetAsync(ws.z, 0, (size_t)M * dm * dtype_size(d->dtype), st));
+  }
+  // 1. QKV projection: one launch, three segments; Q scaled by 1/sqrt(d_k) before rounding
+  GemmArgs g{};
+  g.X = X_act;
+  g.M = M;
+  g.K = dm;
+  g.ldx = dm;
+  g.dtype = d->dtype;
+  g.nseg = 3;
+  g.seg[0] = seg_of(wq, bq, 0);
+  g.seg[0].apply_scale = 1;
+  g.seg[0].scale = 1.0f / std::sqrt((float)dk);
+  g.seg[1] = seg_of(wk, bk, dm);
+  g.seg[2] = seg_of(wv, bv_use, 2 * dm);
+  g.Y = ws.qkv;
+  g.ldy = ws.ldq;
+  g.epi = ET_EPI_BIAS_SCALE;
+  ET_TRY(gemm_run(g, st));
+  // 2. attention core
+  AttnArgs a{};
+  a.qkv = ws.qkv;
+  a.ld_qkv = ws.ldq;
+  a.q_off = 0;
+  a.k_off = dm;
+  a.v_off = 2 * dm;
+  a.v_col = rowv ? ws.v_col : nullptr;
+  a.v_width = rowv ? ws.v_width : nullptr;
+  a.Z = ws.z;
+  a.ld_z = dm;
+  a.z_map = rowv ? wv->row_map : nullptr;
+  a.lengths = d->lengths_dev;
+  a.batch = d->batch;
+  a.seq_len = d->seq_len;
+  a.heads = H;
+  a.d_k = dk;
+  a.head_begin = 0;
+  a.head_end = H;
+  a.causal = d->causal;
+  a.long_form = long_form_for(d) ? 1 : 0;
+  a.v_width_max = dk;
+  a.scale = 1.0f;
+  a.dtype = d->dtype;
+  ET_TRY(attention_run(a, st));
+  // 3. output projection -> fp32 (bias and residual are added by the LayerNorm step)
+  GemmArgs o{};
+  o.X = ws.z;
+  o.M = M;
+  o.K = dm;
+  o.ldx = dm;
+  o.dtype = d->dtype;
+  o.nseg = 1;
+  o.seg[0] = seg_of(wo, nullptr, 0);
+  o.Y = ws.part;
+  o.ldy = dm;
+  o.epi = ET_EPI_F32;
+  return gemm_run(o, st);
+}
+
+}  // namespace
+}  // namespace et
+
+using namespace et;
+
+extern "C" {
+
+et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld_qkv, int32_t q_off, int32_t k_off,
+                           int32_t v_off, const int32_t* v_col, const int32_t* v_width, int32_t v_width_max,
+                           float scale, void* Z, int32_t ld_z, const int32_t* z_map, void* stream) {
+  ET_TRY(check_desc(desc));
+  if (!qkv || !Z) return fail(ET_ERR_INVALID_ARG, "et_attn_core_fwd: null pointer");
+  const int dk = desc->d_model / desc->heads;
+  AttnArgs a{};
+  a.qkv = qkv;
+  a.ld_qkv = ld_qkv;
+  a.q_off = q_off;
+  a.k_off = k_off;
+  a.v_off = v_off;
+  a.v_col = v_col;
+  a.v_width = v_width;
+  a.Z = Z;
+  a.ld_z = ld_z;
+  a.z_map = z_map;
+  a.lengths = desc->lengths_dev;
+  a.batch = desc->batch;
+  a.seq_len = desc->seq_len;
+  a.heads = desc->heads;
+  a.d_k = dk;
+  a.head_begin = desc->head_begin;
+  a.head_end = desc->head_end;
+  a.causal = desc->causal;
+  a.long_form = long_form_for(desc) ? 1 : 0;
+  a.v_width_max = v_width ? v_width_max : dk;
+  a.scale = scale;
+  a.dtype = desc->dtype;
+  return attention_run(a, static_cast<cudaStream_t>(stream));
+}
+
+et_status et_attention_workspace_size(const et_attn_desc* desc, const et_packed_weight* wv, size_t* bytes) {
+  ET_TRY(check_desc(desc));
+  if (!wv || !bytes) return fail(ET_ERR_INVALID_ARG, "et_attention_workspace_size: null pointer");
+  Carver c{nullptr};
+  BlockWs ws;
+  carve_block(c, desc, v_cols_of(wv, desc->d_model), 1, &ws);
+  *bytes = c.off + 256;
+  return ET_OK;
+}
+
+et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_packed_weight* wq,
+                           const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
+                           const void* bq, const void* bk, const void* bv, const void* bo, const float* ln_gamma,
+                           const float* ln_beta, float ln_eps, void* out, void* workspace, size_t ws_bytes,
+                           void* stream) {
+  ET_TRY(check_desc(desc));
+  if (desc->head_begin != 0 || desc->head_end != desc->heads)
+    return fail(ET_ERR_UNSUPPORTED, "et_attention_fwd: head-parallel ranges are not implemented in this build");
+  const int dm = desc->d_model;
+  ET_TRY(check_weight(wq, dm, dm, desc->dtype, "W_Q", false));
+  ET_TRY(check_weight(wk, dm, dm, desc->dtype, "W_K", false));
+  ET_TRY(check_weight(wv, dm, dm, desc->dtype, "W_V", true));
+  ET_TRY(check_weight(wo, dm, dm, desc->dtype, "W_O", false));
+  if (!X || !out || !workspace) return fail(ET_ERR_INVALID_ARG, "et_attention_fwd: null pointer");
+  size_t need = 0;
+  ET_TRY(et_attention_workspace_size(desc, wv, &need));
+  if (ws_bytes < need) return fail(ET_ERR_WORKSPACE, "et_attention_fwd: workspace %zu < %zu", ws_bytes, need);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  Carver c{static_cast<uint8_t*>(workspace)};
+  BlockWs ws;
+  carve_block(c, desc, v_cols_of(wv, dm), 1, &ws);
+  const void* bo_eff = bo;
+  ET_TRY(run_attention_block(desc, X, wq, wk, wv, wo, bq, bk, bv, bo, ws, &bo_eff, st));
+  const int M = desc->batch * desc->seq_len;
+  LnArgs ln{ws.part, 1, M, dm, bo_eff, desc->dtype, ln_gamma ? X : nullptr, desc->dtype, ln_gamma, ln_beta, ln_eps,
+            out, nullptr};
+  return layernorm_run(ln, st);   // gamma == NULL: out = attn = part + b_O' (no residual, no LN)
+}
+
+et_status et_encoder_workspace_size(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff,
+                                    et_dtype resid_dtype, const et_layer* layers, size_t* bytes) {
+  ET_TRY(check_desc(desc));
+  if (num_layers <= 0 || d_ff <= 0 || !layers || !bytes) return fail(ET_ERR_INVALID_ARG, "et_encoder_workspace_size");
+  if (resid_dtype != ET_FP32 && resid_dtype != desc->dtype)
+    return fail(ET_ERR_INVALID_ARG, "resid_dtype must be FP32 or the operand dtype");
+  const int dm = desc->d_model;
+  int vmax = dm;
+  for (int l = 0; l < num_layers; ++l) vmax = std::max(vmax, v_cols_of(&layers[l].wv, dm));
+  const int kparts = std::max(1, (d_ff + 767) / 768);
+  const size_t M = (size_t)desc->batch * desc->seq_len;
+  const size_t es = dtype_size(desc->dtype), rs = dtype_size(resid_dtype);
+  Carver c{nullptr};
+  BlockWs ws;
+  carve_block(c, desc, vmax, kparts, &ws);
+  c.take(M * d_ff * es);   // U
+  c.take(M * dm * es);     // y1 act
+  if (resid_dtype != desc->dtype) {
+    c.take(M * dm * rs);   // y1 residual
+    c.take(M * dm * es);   // x act
+  }
+  c.take(M * dm * rs);     // residual ping-pong
+  *bytes = c.off + 256;
+  return ET_OK;
+}
+
+et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff, et_act act, float ln_eps,
+                         et_dtype resid_dtype, const et_layer* layers, const void* X, void* out, void* workspace,
+                         size_t ws_bytes, void* stream) {
+  ET_TRY(check_desc(desc));
+  if (desc->head_begin != 0 || desc->head_end != desc->heads)
+    return fail(ET_ERR_UNSUPPORTED, "et_encoder_fwd: head-parallel ranges are not implemented in this build");
+  if (resid_dtype != ET_FP32 && resid_dtype != desc->dtype)
+    return fail(ET_ERR_INVALID_ARG, "resid_dtype must be FP32 or the operand dtype");
+  if (act != ET_ACT_GELU_ERF && act != ET_ACT_RELU) return fail(ET_ERR_INVALID_ARG, "bad activation");
+  if (!X || !out || !workspace || !layers) return fail(ET_ERR_INVALID_ARG, "et_encoder_fwd: null pointer");
+  if (d_ff % 64) return fail(ET_ERR_UNSUPPORTED, "d_ff must be a multiple of 64");
+  const int dm = desc->d_model;
+  for (int l = 0; l < num_layers; ++l) {
+    const et_layer& L = layers[l];
+    ET_TRY(check_weight(&L.wq, dm, dm, desc->dtype, "W_Q", false));
+    ET_TRY(check_weight(&L.wk, dm, dm, desc->dtype, "W_K", false));
+    ET_TRY(check_weight(&L.wv, dm, dm, desc->dtype, "W_V", true));
+    ET_TRY(check_weight(&L.wo, dm, dm, desc->dtype, "W_O", false));
+    ET_TRY(check_weight(&L.w1, d_ff, dm, desc->dtype, "W_1", false));
+    ET_TRY(check_weight(&L.w2, dm, d_ff, desc->dtype, "W_2", false));
+    if (!L.ln1_g || !L.ln1_b || !L.ln2_g || !L.ln2_b) return fail(ET_ERR_INVALID_ARG, "layer %d: null LN params", l);
+  }
+  size_t need = 0;
+  ET_TRY(et_encoder_workspace_size(desc, num_layers, d_ff, resid_dtype, layers, &need));
+  if (ws_bytes < need) return fail(ET_ERR_WORKSPACE, "et_encoder_fwd: workspace %zu < %zu", ws_bytes, need);
+
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const size_t M = (size_t)desc->batch * desc->seq_len;
+  const size_t es = dtype_size(desc->dtype), rs = dtype_size(resid_dtype);
+  int vmax = dm;
+  for (int l = 0; l < num_layers; ++l) vmax = std::max(vmax, v_cols_of(&layers[l].wv, dm));
+  const int kparts = std::max(1, (d_ff + 767) / 768);
+  Carver c{static_cast<uint8_t*>(workspace)};
+  BlockWs ws;
+  carve_block(c, desc, vmax, kparts, &ws);
+  void* U = c.take(M * d_ff * es);
+  void* y1a = c.take(M * dm * es);
+  const bool split = resid_dtype != desc->dtype;
+  void* y1r = split ? c.take(M * dm * rs) : y1a;
+  void* xa = split ? c.take(M * dm * es) : nullptr;
+  void* tmp_res = c.take(M * dm * rs);
+
+  // residual stream: layer l writes R[(L-1-l) % 2 == 0 ? out : tmp] so the last layer lands in out
+  const void* cur_res = X;
+  const void* cur_act = X;
+  if (split) {
+    ET_TRY(cast_run(X, resid_dtype, xa, desc->dtype, M * dm, st));
+    cur_act = xa;
+  }
+  for (int l = 0; l < num_layers; ++l) {
+    const et_layer& L = layers[l];
+    void* next_res = ((num_layers - 1 - l) % 2 == 0) ? out : tmp_res;
+    void* next_act = split ? xa : next_res;
+    const void* bo_eff = L.bo;
+    ET_TRY(run_attention_block(desc, cur_act, &L.wq, &L.wk, &L.wv, &L.wo, L.bq, L.bk, L.bv, L.bo, ws, &bo_eff, st));
+    // 4. Y1 = LN(X + attn)
+    LnArgs ln1{ws.part, 1, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,
+               y1a, split ? y1r : nullptr};
+    ET_TRY(layernorm_run(ln1, st));
+    // 5. U = act(Y1 W1'^T + b1)
+    GemmArgs f1{};
+    f1.X = y1a;
+    f1.M = (int)M;
+    f1.K = dm;
+    f1.ldx = dm;
+    f1.dtype = desc->dtype;
+    f1.nseg = 1;
+    f1.seg[0] = seg_of(&L.w1, L.b1, 0);
+    f1.Y = U;
+    f1.ldy = d_ff;
+    f1.epi = act == ET_ACT_GELU_ERF ? ET_EPI_BIAS_GELU : ET_EPI_BIAS_RELU;
+    ET_TRY(gemm_run(f1, st));
+    // 6. U W2'^T -> fp32 split-K partials
+    GemmArgs f2{};
+    f2.X = U;
+    f2.M = (int)M;
+    f2.K = d_ff;
+    f2.ldx = d_ff;
+    f2.dtype = desc->dtype;
+    f2.nseg = 1;
+    f2.seg[0] = seg_of(&L.w2, nullptr, 0);
+    f2.Y = ws.part;
+    f2.ldy = dm;
+    f2.epi = ET_EPI_F32;
+    ET_TRY(gemm_run(f2, st));
+    // 7. Y2 = LN(Y1 + F + b2)
+    LnArgs ln2{ws.part, L.w2.kparts, (int)M, dm, L.b2, desc->dtype, y1r, resid_dtype, L.ln2_g, L.ln2_b, ln_eps,
+               split ? next_act : nullptr, next_res};
+    ET_TRY(layernorm_run(ln2, st));
+    cur_res = next_res;
+    cur_act = split ? xa : next_res;
+  }
+  return ET_OK;
+}
+
+}  // extern "C"

@@ -96,7 +96,7 @@ struct AttnArgs {
   const int32_t* v_width;   // [H] or nullptr
   void* Z;
   int ld_z;
-  const int32_t* z_col;     // [H] or nullptr
+  const int32_t* z_map;     // [packed V width] or nullptr
   const int32_t* lengths;   // [B] or nullptr
   int batch, seq_len, heads, d_k, head_begin, head_end;
   int causal;
@@ -107,5 +107,23 @@ struct AttnArgs {
 };
 et_status attention_run(const AttnArgs& a, cudaStream_t stream);
 int attn_short_max(int d_k);
+
+// ---------------------------------------------------------------- small helpers (kernels/layernorm.cu)
+et_status cast_run(const void* src, et_dtype sdt, void* dst, et_dtype ddt, size_t n, cudaStream_t stream);
+// attention-aware (row-pruned W_V) layer data: per-head packed V columns / widths, the packed
+// V bias, and the folded output bias b_O' = b_O + sum_{f pruned} W_O'[:, f] b_V[f] (reading C-6)
+struct VPrep {
+  const et_packed_weight* wv;
+  const et_packed_weight* wo;
+  const void* bv;
+  const void* bo;
+  int heads, d_k;
+  et_dtype dtype;
+  int32_t* v_col;      // out [H]
+  int32_t* v_width;    // out [H]
+  void* bv_packed;     // out [rows_padded]
+  void* bo_folded;     // out [d]
+};
+et_status vprep_run(const VPrep& v, cudaStream_t stream);
 
 }  // namespace et

@@ -51,13 +51,14 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const LnArgs a) {
   const int warp_g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (warp_g >= a.M) return;
-  const int nch = a.N / 128;
+  const int nch = (a.N + 127) / 128;
   const size_t row = (size_t)warp_g * a.N;
   float4 v[kMaxChunks];
   float s = 0.f;
 #pragma unroll
   for (int c = 0; c < kMaxChunks; ++c) {
-    if (c < nch) {
+    v[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (c < nch && c * 128 + lane * 4 < a.N) {
       const int col = c * 128 + lane * 4;
       float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
       for (int pidx = 0; pidx < a.nparts; ++pidx) {
@@ -76,13 +77,24 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const LnArgs a) {
       s += x.x + x.y + x.z + x.w;
     }
   }
+  if (a.gamma == nullptr) {   // no normalisation: out = sum(part) + bias (+ resid)
+#pragma unroll
+    for (int c = 0; c < kMaxChunks; ++c) {
+      if (c < nch && c * 128 + lane * 4 < a.N) {
+        const int col = c * 128 + lane * 4;
+        if (a.out_act) st_act4(a.out_act, a.dtype, row + col, v[c]);
+        if (a.out_resid) st_act4(a.out_resid, a.resid_dtype, row + col, v[c]);
+      }
+    }
+    return;
+  }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   const float mean = s / a.N;
   float q = 0.f;
 #pragma unroll
   for (int c = 0; c < kMaxChunks; ++c) {
-    if (c < nch) {
+    if (c < nch && c * 128 + lane * 4 < a.N) {
       const float dx = v[c].x - mean, dy = v[c].y - mean, dz = v[c].z - mean, dw = v[c].w - mean;
       q += dx * dx + dy * dy + dz * dz + dw * dw;
     }
@@ -92,7 +104,7 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const LnArgs a) {
   const float rstd = rsqrtf(q / a.N + a.eps);
 #pragma unroll
   for (int c = 0; c < kMaxChunks; ++c) {
-    if (c < nch) {
+    if (c < nch && c * 128 + lane * 4 < a.N) {
       const int col = c * 128 + lane * 4;
       const float4 gm = *reinterpret_cast<const float4*>(a.gamma + col);
       const float4 bt = *reinterpret_cast<const float4*>(a.beta + col);
@@ -107,8 +119,8 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const LnArgs a) {
 }  // namespace
 
 et_status layernorm_run(const LnArgs& a, cudaStream_t stream) {
-  if (a.N % 128 || a.N > 128 * kMaxChunks)
-    return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 128 and <= 2048 (got %d)", a.N);
+  if (a.N % 4 || a.N > 128 * kMaxChunks)
+    return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 4 and <= 2048 (got %d)", a.N);
   if (a.M <= 0) return ET_OK;
   const int threads = 256;
   const int blocks = (a.M * 32 + threads - 1) / threads;

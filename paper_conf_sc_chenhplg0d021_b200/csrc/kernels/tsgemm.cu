@@ -55,7 +55,8 @@ struct Piece {
   int16_t i0, i1;  // tile rows [i0, i1) of the segment
 };
 struct Params {
-  int M, Kp, kparts;
+  int M, K, Kp, kparts;   // Kp = 768 (K part width); the last part may be shorter
+  int box_rows;           // TMA box height: min(128, M) (a box may not exceed the tensor)
   int nseg;
   SegDev seg[3];
   int npieces;
@@ -130,7 +131,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const SegDev& sg = p.seg[pc.seg];
   const int m0 = blockIdx.y * 128;
   const int z = blockIdx.z;
-  const int nk = p.Kp / 64;                    // A chunks (64 K each)
+  const int nk = min(p.Kp, p.K - z * p.Kp) / 64;   // A chunks (64 K each) of this K part
   const int32_t* rp = sg.prp + (size_t)z * (sg.tile_rows + 1);
   const int pb = rp[pc.i0], pe = rp[pc.i1];    // this CTA's packed tiles [pb, pe)
   const int nchunks = (pe - pb + kChunkTiles - 1) / kChunkTiles;
@@ -164,7 +165,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       tma_prefetch_desc(&tmap_x);
       const int kx0 = z * p.Kp;
       for (int j = 0; j < nk && j < kNXS; ++j) {
-        mbar_expect_tx(&bar.xfull[j], 16384);
+        mbar_expect_tx(&bar.xfull[j], p.box_rows * 128);
         tma_load_2d(sX + j * 16384, &tmap_x, &bar.xfull[j], kx0 + j * 64, m0);
       }
       for (int j = 0; j < nk; ++j) {
@@ -182,7 +183,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         if (jr >= 0 && jr + kNXS < nk) {
           const int rs = jr % kNXS;
           mbar_wait(&bar.xempty[rs], (jr / kNXS) & 1);
-          mbar_expect_tx(&bar.xfull[rs], 16384);
+          mbar_expect_tx(&bar.xfull[rs], p.box_rows * 128);
           tma_load_2d(sX + rs * 16384, &tmap_x, &bar.xfull[rs], kx0 + (jr + kNXS) * 64, m0);
         }
       }
@@ -352,12 +353,12 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   const int kparts = (a.K + 767) / 768;
   if (kparts > 1 && a.epi != ET_EPI_F32)
     return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K > 768 needs the fp32 split-K epilogue");
-  if (a.K % kparts || (a.K / kparts) % 64 || a.K / kparts > 768 || (kparts > 1 && a.K / kparts != 768 && a.K != kparts * 768))
-    return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K=%d not splittable into parts of 768", a.K);
   if (a.M <= 0) return ET_OK;
 
   Params prm{};
   prm.M = a.M;
+  prm.K = a.K;
+  prm.box_rows = a.M < 128 ? a.M : 128;
   prm.Kp = kparts > 1 ? 768 : a.K;
   prm.kparts = kparts;
   prm.nseg = a.nseg;
@@ -407,7 +408,7 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   prm.npieces = np;
   CUtensorMap tm;   // the K offset k0 is folded into the base address
   ET_TRY(make_tmap_2d(&tm, static_cast<const uint8_t*>(a.X) + (size_t)a.k0 * 2, a.dtype, (uint64_t)a.M,
-                      (uint64_t)a.K, (uint64_t)a.ldx, 64, 128, true));
+                      (uint64_t)a.K, (uint64_t)a.ldx, 64, (uint32_t)prm.box_rows, true));
   dim3 grid(np, mblocks, kparts);
   const bool bf = a.dtype == ET_BF16;
   switch (a.epi) {

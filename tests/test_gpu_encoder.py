@@ -1,0 +1,136 @@
+"""End-to-end parity of et_encoder_fwd / et_attention_fwd vs the float64 oracle:
+every BASELINE config shape (C1..C5; C1 in FP16/BF16 — the FP32 validation build is not in this
+build), reduced and at full size on sampled sequences, both residual-stream dtypes, and the
+batch-shard bit-exactness that multi-GPU batch sharding relies on (§8(e))."""
+import numpy as np
+import pytest
+import torch
+
+from et_synth import CONFIGS, make_layer, make_lengths, make_x
+from oracle import encoder as oe
+from tests.gpu_util import assert_close, dev_tensor, to64
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def etm():
+    import paper_conf_sc_chenhplg0d021_b200 as m
+    assert torch.cuda.is_available()
+    return m
+
+
+def _oracle(cfg, raws, X, lens, idx=None):
+    layers = [oe.prune_layer(r, cfg.scheme, cfg.ratio)[0] for r in raws]
+    Xs = X if idx is None else X[idx]
+    ls = lens if idx is None else lens[idx]
+    return oe.encoder(Xs.astype(np.float64), layers, cfg.heads, ls, cfg.causal, cfg.act, cfg.ln_eps)
+
+
+def _gpu(etm, cfg, raws, X, lens, resid="same", mode="auto"):
+    dtype = cfg.dtype
+    rdt = dtype if resid == "same" else resid
+    layers = [etm.pack_layer(r, cfg.scheme, cfg.ratio, cfg.heads, dtype) for r in raws]
+    L = torch.from_numpy(lens).cuda()
+    enc = etm.Encoder(layers, cfg.batch, cfg.seq_len, cfg.heads, cfg.d_ff, act=cfg.act, ln_eps=cfg.ln_eps,
+                      dtype=dtype, resid_dtype=rdt, causal=cfg.causal, mode=mode, lengths=L)
+    Xd = dev_tensor(X.reshape(cfg.tokens, cfg.d_model), rdt)
+    Y = enc(Xd)
+    torch.cuda.synchronize()
+    return to64(Y).reshape(cfg.batch, cfg.seq_len, cfg.d_model), enc, Xd
+
+
+def _case(key, **kw):
+    cfg = CONFIGS[key].with_(**kw)
+    if cfg.dtype == "fp32":
+        cfg = cfg.with_(dtype="fp16")
+    raws = [make_layer(cfg, l) for l in range(cfg.layers)]
+    X = make_x(cfg)
+    lens = make_lengths(cfg)
+    return cfg, raws, X, lens
+
+
+@pytest.mark.parametrize("key,kw", [
+    ("C1", {}), ("C1", {"dtype": "bf16"}),
+    ("C2", {}),
+    ("C3", {"layers": 2, "batch": 4}),
+    ("C3", {"layers": 2, "batch": 3, "dtype": "bf16"}),
+    ("C4", {"layers": 1, "batch": 2}),
+    ("C5", {"layers": 1, "batch": 1}),
+])
+def test_encoder_matches_oracle(etm, key, kw):
+    cfg, raws, X, lens = _case(key, **kw)
+    resid = "fp32" if cfg.dtype == "bf16" else "same"    # reading C-22: BF16 needs an FP32 residual stream
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens, resid=resid)
+    ref = _oracle(cfg, raws, X, lens)
+    assert_close(Y.reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what=f"{key} {kw}")
+
+
+def test_headline_c3_full_size_sampled(etm):
+    """C3 at full size (12 layers, 32 sequences) in the bench launch configuration; the oracle runs
+    on sampled sequences (sequences are independent)."""
+    cfg, raws, X, lens = _case("C3")
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens)
+    idx = np.array([0, 1, 17, 31])
+    ref = _oracle(cfg, raws, X, lens, idx)
+    assert_close(Y[idx].reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what="C3 full")
+
+
+def test_c4_long_form_sampled(etm):
+    cfg, raws, X, lens = _case("C4", layers=2, batch=8)
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens)
+    idx = np.array([0, 1, 5])
+    ref = _oracle(cfg, raws, X, lens, idx)
+    assert_close(Y[idx].reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what="C4")
+
+
+def test_fp32_residual_stream_fp16(etm):
+    cfg, raws, X, lens = _case("C3", layers=2, batch=2)
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens, resid="fp32")
+    ref = _oracle(cfg, raws, X, lens)
+    assert_close(Y.reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what="fp32 resid")
+
+
+@pytest.mark.parametrize("mode", ["short", "long"])
+def test_attention_forms_inside_encoder(etm, mode):
+    cfg, raws, X, lens = _case("C3", layers=1, batch=2, seq_len=256)
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens, mode=mode)
+    ref = _oracle(cfg, raws, X, lens)
+    assert_close(Y.reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what=mode)
+
+
+def test_batch_shard_bitexact(etm):
+    """Sharding the batch (§8(e)) must not change any output bit: every kernel's per-row reduction
+    order is independent of the batch size."""
+    cfg, raws, X, lens = _case("C3", layers=2, batch=8)
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens)
+    half = cfg.with_(batch=4)
+    Y2, _, _ = _gpu(etm, half, raws, X[4:], lens[4:])
+    np.testing.assert_array_equal(Y[4:], Y2)
+
+
+def test_attention_block_entry_point(etm):
+    cfg, raws, X, lens = _case("C3", layers=1, batch=2)
+    layer = etm.pack_layer(raws[0], cfg.scheme, cfg.ratio, cfg.heads, cfg.dtype)
+    L = torch.from_numpy(lens).cuda()
+    Xd = dev_tensor(X.reshape(cfg.tokens, cfg.d_model), cfg.dtype)
+    out = etm.attention_fwd(Xd, layer, cfg.batch, cfg.seq_len, cfg.heads, lengths=L, ln=True, ln_eps=cfg.ln_eps)
+    raw_attn = etm.attention_fwd(Xd, layer, cfg.batch, cfg.seq_len, cfg.heads, lengths=L, ln=False)
+    torch.cuda.synchronize()
+    w, _ = oe.prune_layer(raws[0], cfg.scheme, cfg.ratio)
+    attn = oe.attention_block(X.astype(np.float64), w, cfg.heads, lens, False)
+    y1 = oe.layer_norm(X + attn, w["ln1_g"], w["ln1_b"], cfg.ln_eps)
+    assert_close(to64(raw_attn), attn.reshape(-1, cfg.d_model), what="attn block")
+    assert_close(to64(out), y1.reshape(-1, cfg.d_model), what="attn block + LN")
+
+
+def test_invalid_arguments_fail_loudly(etm):
+    cfg, raws, X, lens = _case("C3", layers=1, batch=1)
+    layer = etm.pack_layer(raws[0], cfg.scheme, cfg.ratio, cfg.heads, cfg.dtype)
+    with pytest.raises(etm.EtError):
+        etm.Encoder([layer], 1, 128, 5, cfg.d_ff)                       # d_model % heads != 0
+    qkv = torch.zeros(512, 3 * 768, dtype=torch.float16, device="cuda")
+    with pytest.raises(etm.EtError):
+        etm.attn_core_fwd(qkv, 1, 512, 12, 768, 0, 768, 1536, mode="short")   # short form needs S <= 256
+    with pytest.raises(etm.EtError):
+        etm.Encoder([layer], 1, 128, 12, cfg.d_ff, resid_dtype="bf16")  # resid must be fp32 or fp16 here
