@@ -1,0 +1,415 @@
+#!/usr/bin/env python
+"""bench.py — BERT-base encoder throughput of the B200-native E.T. hot path (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C3]
+
+One step = one full forward of the workload's encoder stack over one batch of synthetic input
+(SURVEY §8(a) rows a2-a7), through the library's public entry point et_encoder_fwd.
+
+Workload (N=1): configs[2] = C3, BERT-base (12 layers, 12 heads, d_model 768, d_ff 3072), seq_len 128,
+batch 32, 80 % tensor-tile pruning (16x16), FP16 — the configuration the metric is quoted on.
+Multi-GPU (torchrun, one rank per GPU): the batch is sharded, every rank runs its own 32 sequences
+(weak scaling, no collective on the data path; sequences are independent).
+
+Timing: W untimed warm-up steps; then K steps, each bracketed by CUDA events on the launching stream,
+L2 flushed (256 MiB write) before every step outside the events; barrier + synchronize around the
+whole region; value = sequences of all ranks / max over ranks of the summed step time.  Per-kernel
+times come from the library's trace events recorded live in the same timed steps (roofline).
+`e2e` repeats the measurement through the same call with pinned-host input / output copies inside
+the timed region.  `cpu_baseline`: the float64 CPU oracle (tests' reference; never the product path)
+on a bounded sample, rank 0 at N=1 only.  `--impl reference`: that oracle as the reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "BERT-base encoder seqs/sec @seq128, 80% tile-pruned; % tensor-pipe/HBM roofline"
+KIND_NAMES = ["qkv_gemm", "attention", "oproj_gemm", "ln1", "ffn1_gemm", "ffn2_gemm", "ln2", "aux"]
+SPEC_TC_TFLOPS = 2250.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="C3")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the cpu_baseline sample")
+    return ap.parse_args()
+
+
+def peaks():
+    p = {"hbm_gbs": 6482.1, "bf16_tflops": 1637.3, "bf16_tflops_sustained": 1384.3, "src": "MEASURED_PEAKS.json"}
+    f = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(f):
+        with open(f) as fh:
+            m = json.load(fh)
+        for k in ("hbm_gbs", "bf16_tflops", "bf16_tflops_sustained"):
+            if k in m:
+                p[k] = float(m[k])
+    else:
+        p.update({"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+                  "src": "fallback (B200_PROFILING.md)"})
+    return p
+
+
+# ------------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons, pw = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+                pw.append(float(f[3]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        load = [s for s in sm if s > 300] or sm
+        return {"sm_mhz": statistics.median(load) if load else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm), "power_w_max": max(pw) if pw else None}
+
+
+# ------------------------------------------------------------------------------------------ roofline model
+def kernel_model(cfg, nnz: dict, kparts2: int, es: int, resid_es: int):
+    """Algorithmic bytes and (effective) FLOPs of ONE launch of each kernel kind for one layer of
+    `cfg`.  nnz: kept 16x16 tiles per matrix."""
+    M, d, f, H, S, B = cfg.tokens, cfg.d_model, cfg.d_ff, cfg.heads, cfg.seq_len, cfg.batch
+    dk = d // H
+    t = 512   # bytes per packed 16x16 fp16/bf16 tile
+    mm = lambda n: 2.0 * M * 256 * n          # one MMA tile = 16x16 weights against M tokens
+    pairs = B * H * (S * (S + 1) / 2 if cfg.causal else S * S)
+    return {
+        "qkv_gemm": (M * d * es + (nnz["wq"] + nnz["wk"] + nnz["wv"]) * t + M * 3 * d * es,
+                     mm(nnz["wq"] + nnz["wk"] + nnz["wv"])),
+        "attention": (M * 3 * d * es + M * d * es, 4.0 * pairs * dk),
+        "oproj_gemm": (M * d * es + nnz["wo"] * t + M * d * 4, mm(nnz["wo"])),
+        "ln1": (M * d * 4 + M * d * resid_es + M * d * es, 0.0),
+        "ffn1_gemm": (M * d * es + nnz["w1"] * t + M * f * es, mm(nnz["w1"])),
+        "ffn2_gemm": (M * f * es + nnz["w2"] * t + kparts2 * M * d * 4, mm(nnz["w2"])),
+        "ln2": (kparts2 * M * d * 4 + M * d * resid_es + M * d * resid_es, 0.0),
+    }
+
+
+def eff_flops_per_step(cfg, nnz_layers):
+    """North-star numerator: FLOPs on kept tiles + attention on unmasked pairs, all layers."""
+    tot = 0.0
+    M, H, S, B, d = cfg.tokens, cfg.heads, cfg.seq_len, cfg.batch, cfg.d_model
+    pairs = B * H * (S * (S + 1) / 2 if cfg.causal else S * S)
+    for nz in nnz_layers:
+        tot += 2.0 * M * 256 * sum(nz.values()) + 4.0 * pairs * (d // H)
+    return tot
+
+
+# ------------------------------------------------------------------------------------------ CPU oracle
+def oracle_seqs_per_s(cfg, raws, X, lens, budget_s: float, chunk: int):
+    """Time the float64 CPU oracle (as it stands) on chunks of `chunk` sequences until the budget."""
+    from oracle import encoder as oe
+    layers = [oe.prune_layer(r, cfg.scheme, cfg.ratio)[0] for r in raws]
+    done, t0 = 0, time.perf_counter()
+    while True:
+        i0 = done % cfg.batch
+        idx = np.arange(i0, i0 + chunk) % cfg.batch
+        oe.encoder(X[idx].astype(np.float64), layers, cfg.heads, lens[idx], cfg.causal, cfg.act, cfg.ln_eps)
+        done += chunk
+        el = time.perf_counter() - t0
+        if el >= budget_s:
+            return done / el, done, el
+
+
+def cpu_threads():
+    try:
+        from threadpoolctl import threadpool_info
+        n = [i.get("num_threads") for i in threadpool_info() if i.get("user_api") == "blas"]
+        if n:
+            return int(max(n))
+    except Exception:
+        pass
+    return os.cpu_count()
+
+
+def reference_arm(args):
+    """--impl reference: the CPU oracle on the same config/metric (bounded sample per step)."""
+    from et_synth import CONFIGS, make_layer, make_lengths, make_x
+    cfg = CONFIGS[args.config]
+    raws = [make_layer(cfg, l) for l in range(cfg.layers)]
+    X = make_x(cfg)
+    lens = make_lengths(cfg, ragged=False)
+    from oracle import encoder as oe
+    layers = [oe.prune_layer(r, cfg.scheme, cfg.ratio)[0] for r in raws]
+    per_step = 2
+    for w in range(args.warmup):
+        idx = np.arange(w * per_step, (w + 1) * per_step) % cfg.batch
+        oe.encoder(X[idx].astype(np.float64), layers, cfg.heads, lens[idx], cfg.causal, cfg.act, cfg.ln_eps)
+    t0 = time.perf_counter()
+    for s in range(args.steps):
+        idx = np.arange(s * per_step, (s + 1) * per_step) % cfg.batch
+        oe.encoder(X[idx].astype(np.float64), layers, cfg.heads, lens[idx], cfg.causal, cfg.act, cfg.ln_eps)
+    el = time.perf_counter() - t0
+    v = per_step * args.steps / el
+    sample = f"{per_step} sequences of {args.config} per step (float64 numpy, all {cfg.layers} layers)"
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "seqs/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * el / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload_name(cfg), "global_batch": cfg.batch, "seq_len": cfg.seq_len},
+            "cpu_baseline": {"value": v, "unit": "seqs/s", "cores": cpu_threads(), "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": v, "unit": "seqs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def workload_name(cfg):
+    return (f"{cfg.name}: {cfg.layers}-layer encoder, {cfg.heads} heads, d_model {cfg.d_model}, d_ff {cfg.d_ff}, "
+            f"seq_len {cfg.seq_len}, {cfg.ratio:.0%} {cfg.scheme} pruning (16x16 tiles), {cfg.dtype}, "
+            f"{'causal' if cfg.causal else 'padding'} mask")
+
+
+# ------------------------------------------------------------------------------------------ our arm
+def our_arm(args):
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py: no CUDA device (this benchmark has no CPU fallback)")
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_sc_chenhplg0d021_b200 as et
+    from et_synth import CONFIGS, make_layer, make_lengths, make_x
+
+    base = CONFIGS[args.config]
+    cfg = base                                   # per-rank shard: the config's batch (weak scaling)
+    gcfg = base.with_(batch=base.batch * world)  # the global batch, generated identically everywhere
+    dtype = cfg.dtype if cfg.dtype != "fp32" else "fp16"
+    raws = [make_layer(cfg, l) for l in range(cfg.layers)]
+    Xg = make_x(gcfg)
+    X = Xg[rank * cfg.batch:(rank + 1) * cfg.batch]
+    lens = make_lengths(cfg, ragged=False)
+
+    layers = [et.pack_layer(r, cfg.scheme, cfg.ratio, cfg.heads, dtype) for r in raws]
+    nnz_layers = [{n: l.packed[n].c.ntiles for n in ("wq", "wk", "wv", "wo", "w1", "w2")} for l in layers]
+    L = torch.from_numpy(lens).cuda()
+    enc = et.Encoder(layers, cfg.batch, cfg.seq_len, cfg.heads, cfg.d_ff, act=cfg.act, ln_eps=cfg.ln_eps,
+                     dtype=dtype, resid_dtype=dtype, causal=cfg.causal, mode=cfg.attn_mode, lengths=L)
+    tdt = et.torch_dtype(dtype)
+    Xd = torch.from_numpy(np.ascontiguousarray(X.reshape(cfg.tokens, cfg.d_model))).cuda().to(tdt)
+    out = torch.empty_like(Xd)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+
+    for _ in range(max(args.warmup, 3)):
+        enc(Xd, out)
+    torch.cuda.synchronize()
+
+    # ---------------- timed region: K steps, per-step events, L2 flushed between steps
+    K = args.steps
+    cap = K * (len(layers) * 8 + 4) + 8
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    clk = ClockSampler(local)
+    barrier()
+    torch.cuda.synchronize()
+    clk.start()
+    launches0 = et._lib.et_launch_count()
+    et._check(et._lib.et_trace_begin(cap))
+    for s in range(K):
+        flush.fill_(float(s))
+        ev[s][0].record(stream)
+        enc(Xd, out)
+        ev[s][1].record(stream)
+    n_int = __import__("ctypes").c_int32()
+    et._check(et._lib.et_trace_end(__import__("ctypes").byref(n_int)))
+    launches = et._lib.et_launch_count() - launches0
+    torch.cuda.synchronize()
+    barrier()
+    clocks = clk.stop()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    t_local = sum(step_ms) / 1e3
+    # per-kernel trace
+    import ctypes
+    kind = ctypes.c_int32()
+    ms = ctypes.c_float()
+    per_kind = {}
+    for i in range(n_int.value):
+        et._check(et._lib.et_trace_get(i, ctypes.byref(kind), ctypes.byref(ms)))
+        if kind.value < len(KIND_NAMES):
+            per_kind.setdefault(KIND_NAMES[kind.value], []).append(ms.value)
+
+    # ---------------- end to end: pinned host input -> device, forward, device -> pinned host output
+    e2e = None
+    if not args.no_e2e:
+        Xh = torch.from_numpy(np.ascontiguousarray(X.reshape(cfg.tokens, cfg.d_model))).to(tdt).pin_memory()
+        Oh = torch.empty_like(Xh).pin_memory()
+        Xin = torch.empty_like(Xd)
+        eev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+        for _ in range(2):
+            Xin.copy_(Xh, non_blocking=True)
+            enc(Xin, out)
+            Oh.copy_(out, non_blocking=True)
+        torch.cuda.synchronize()
+        barrier()
+        for s in range(K):
+            flush.fill_(float(s))
+            eev[s][0].record(stream)
+            Xin.copy_(Xh, non_blocking=True)
+            enc(Xin, out)
+            Oh.copy_(out, non_blocking=True)
+            eev[s][1].record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        e2e_local = sum(a.elapsed_time(b) for a, b in eev) / 1e3
+        e2e = {"t": e2e_local, "h2d": Xh.numel() * Xh.element_size() + L.numel() * 0,
+               "d2h": Oh.numel() * Oh.element_size()}
+
+    # ---------------- max over ranks
+    t_max = t_local
+    e2e_max = e2e["t"] if e2e else None
+    if dist is not None:
+        tt = torch.tensor([t_local, e2e_max or 0.0], dtype=torch.float64, device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_max, e2e_max = float(tt[0]), (float(tt[1]) if e2e else None)
+
+    if rank == 0:
+        pk = peaks()
+        total_seqs = cfg.batch * world * K
+        value = total_seqs / t_max
+        es = 2
+        model = kernel_model(cfg, nnz_layers[0], layers[0].packed["w2"].c.kparts, es, es)
+        # dominant kernel: largest share of the traced step time
+        tot = {k: sum(v) for k, v in per_kind.items()}
+        dom = max(tot, key=tot.get) if tot else None
+        roof = None
+        if dom and dom in model:
+            avg_s = statistics.mean(per_kind[dom]) / 1e3
+            nbytes, nflops = model[dom]
+            t_hbm = nbytes / (pk["hbm_gbs"] * 1e9)
+            t_tc = nflops / (pk["bf16_tflops_sustained"] * 1e12)
+            traffic = None
+            tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+            if os.path.exists(tf):
+                with open(tf) as fh:
+                    traffic = json.load(fh).get(dom)
+            if t_tc > t_hbm:
+                ach = nflops / avg_s / 1e12
+                roof = {"bound": "tensor", "achieved": ach, "peak": pk["bf16_tflops_sustained"], "unit": "TFLOP/s",
+                        "frac": ach / pk["bf16_tflops_sustained"], "traffic": traffic, "kernel": dom,
+                        "algorithmic_flops_per_launch": nflops, "avg_launch_ms": avg_s * 1e3,
+                        "peak_src": pk["src"] + " bf16_tflops_sustained (fp16 dense = bf16 dense)"}
+            else:
+                ach = nbytes / avg_s / 1e9
+                roof = {"bound": "hbm", "achieved": ach, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                        "frac": ach / pk["hbm_gbs"], "traffic": traffic, "kernel": dom,
+                        "algorithmic_bytes_per_launch": nbytes, "avg_launch_ms": avg_s * 1e3,
+                        "peak_src": pk["src"] + " hbm_gbs"}
+        share = {k: round(v / sum(tot.values()), 4) for k, v in tot.items()} if tot else {}
+        kern_ms = {k: round(statistics.mean(v), 5) for k, v in per_kind.items()}
+        eflops = eff_flops_per_step(cfg, nnz_layers) * world
+        ns = {"eff_tflops": eflops * K / t_max / 1e12}
+        ns["frac_of_measured_tc"] = ns["eff_tflops"] / pk["bf16_tflops"]
+        ns["frac_of_spec_tc"] = ns["eff_tflops"] / SPEC_TC_TFLOPS
+        line = {
+            "metric": METRIC, "value": value, "unit": "seqs/s", "n_gpus": world, "steps": K,
+            "warmup": max(args.warmup, 3), "ms_per_step": 1e3 * t_max / K, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": dtype, "data": "synthetic",
+            "config": {"workload": workload_name(cfg), "global_batch": cfg.batch * world,
+                       "seq_len": cfg.seq_len, "per_gpu_batch": cfg.batch,
+                       "parallelism": f"dp{world} (batch sharded, no data-path collective)",
+                       "l2": "flushed before every timed step (256 MiB write, outside the events)",
+                       "residual_stream": dtype, "attention_form": "short" if cfg.seq_len <= 256 else "long"},
+            "roofline": roof,
+            "kernel_ms": kern_ms, "kernel_share": share,
+            "north_star": ns,
+            "gpu_launches": int(launches),
+            "clocks": clocks,
+            "step_ms_p50": statistics.median(step_ms),
+        }
+        if e2e:
+            line["e2e"] = {"value": total_seqs / e2e_max, "unit": "seqs/s", "h2d_bytes_per_step": e2e["h2d"],
+                           "d2h_bytes_per_step": e2e["d2h"]}
+        if world == 1 and not args.no_cpu_baseline:
+            v, n, el = oracle_seqs_per_s(cfg, raws, X, lens, args.cpu_seconds, chunk=2)
+            line["cpu_baseline"] = {"value": v, "unit": "seqs/s", "cores": cpu_threads(), "kind": "oracle",
+                                    "sample": f"{n} sequences of {args.config} (all {cfg.layers} layers, float64 "
+                                              f"numpy oracle, {el:.1f} s)"}
+        print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.impl == "reference":
+        if int(os.environ.get("RANK", "0")) == 0:
+            reference_arm(args)
+        return
+    if args.gpus > 1 and world == 1 and "RANK" not in os.environ:
+        # launched directly with --gpus N: re-launch one process per GPU through torchrun
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", "29517", __file__] + sys.argv[1:]
+        raise SystemExit(subprocess.call(cmd))
+    our_arm(args)
+
+
+if __name__ == "__main__":
+    main()

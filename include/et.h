@@ -221,6 +221,25 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
                          et_dtype resid_dtype, const et_layer* layers_host, const void* X, void* out,
                          void* workspace, size_t ws_bytes, void* stream);
 
+/* ------------------------------------------------------------------------------------------
+ * Tracing (calling thread only): while enabled, the forward entry points record a CUDA event on
+ * the caller's stream before every kernel they launch (and one after the last), tagged with the
+ * step kind, so that per-kernel device time can be read back after the stream is synchronised.
+ * Event handles are created lazily by the library (no device memory).  Recording stops silently
+ * once `capacity` marks have been taken.
+ * ------------------------------------------------------------------------------------------ */
+typedef enum {
+  ET_K_QKV = 0, ET_K_ATTN = 1, ET_K_OPROJ = 2, ET_K_LN1 = 3, ET_K_FFN1 = 4, ET_K_FFN2 = 5, ET_K_LN2 = 6,
+  ET_K_AUX = 7, ET_K_END = 8
+} et_kernel_kind;
+et_status et_trace_begin(int32_t capacity);
+/* Stop recording; *n_intervals = number of recorded kernel intervals. */
+et_status et_trace_end(int32_t* n_intervals);
+/* Interval i (after synchronising the stream): its kind and device milliseconds. */
+et_status et_trace_get(int32_t i, int32_t* kind, float* ms);
+/* Number of library kernels launched by this thread since process start (launch accounting). */
+int64_t et_launch_count(void);
+
 /* Diagnostics (not part of the metric): tcgen05 probe (profiles/r01/M1_tcgen05_probe.md). */
 int et_diag_mma_probe(const void* A, const void* B, float* D, int N, int a_mode, int b_mode, int iters, int n_acc,
                       int issue_mode, long long* cycles, int grid, void* stream);

@@ -366,3 +366,11 @@ class Encoder:
 def encoder_fwd(X: torch.Tensor, layers: list, batch: int, seq_len: int, heads: int, d_ff: int, **kw):
     """One-shot et_encoder_fwd (allocates the workspace; use Encoder for repeated calls)."""
     return Encoder(layers, batch, seq_len, heads, d_ff, **kw)(X)
+
+
+# ------------------------------------------------------------------------------------------ tracing
+_sig("et_trace_begin", ctypes.c_int, [_i32])
+_sig("et_trace_end", ctypes.c_int, [ctypes.POINTER(_i32)])
+_sig("et_trace_get", ctypes.c_int, [_i32, ctypes.POINTER(_i32), ctypes.POINTER(_f32)])
+_sig("et_launch_count", ctypes.c_int64, [])
+SYMBOLS += ["et_trace_begin", "et_trace_end", "et_trace_get", "et_launch_count"]

@@ -5,6 +5,7 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include "internal.h"
 
@@ -31,6 +32,32 @@ et_status fail(et_status s, const char* fmt, ...) {
   return s;
 }
 
+// ---------------------------------------------------------------- tracing
+struct Trace {
+  bool on = false;
+  int capacity = 0, n = 0;
+  std::vector<cudaEvent_t> ev;
+  std::vector<int> kind;
+};
+static thread_local Trace g_trace;
+static thread_local long long g_launches = 0;
+
+void count_launch() { ++g_launches; }
+
+void trace_mark(int kind, cudaStream_t stream) {
+  Trace& t = g_trace;
+  if (!t.on || t.n >= t.capacity) return;
+  if ((int)t.ev.size() <= t.n) {
+    cudaEvent_t e;
+    if (cudaEventCreate(&e) != cudaSuccess) return;
+    t.ev.push_back(e);
+    t.kind.push_back(0);
+  }
+  cudaEventRecord(t.ev[t.n], stream);
+  t.kind[t.n] = kind;
+  ++t.n;
+}
+
 static bool valid_dtype(et_dtype d) { return d == ET_FP16 || d == ET_BF16 || d == ET_FP32; }
 
 static int units_of(int rows, int cols, et_pattern pat, int r, int c) {
@@ -49,6 +76,32 @@ extern "C" {
 
 const char* et_last_error(void) { return g_err.c_str(); }
 const char* et_version(void) { return "et-b200 0.1 (sm_100a)"; }
+
+et_status et_trace_begin(int32_t capacity) {
+  if (capacity < 2) return fail(ET_ERR_INVALID_ARG, "et_trace_begin: capacity < 2");
+  g_trace.on = true;
+  g_trace.capacity = capacity;
+  g_trace.n = 0;
+  return ET_OK;
+}
+
+et_status et_trace_end(int32_t* n_intervals) {
+  g_trace.on = false;
+  if (n_intervals) *n_intervals = g_trace.n > 0 ? g_trace.n - 1 : 0;
+  return ET_OK;
+}
+
+et_status et_trace_get(int32_t i, int32_t* kind, float* ms) {
+  if (i < 0 || i + 1 >= g_trace.n) return fail(ET_ERR_INVALID_ARG, "et_trace_get: index out of range");
+  if (kind) *kind = g_trace.kind[i];
+  if (ms) {
+    cudaError_t e = cudaEventElapsedTime(ms, g_trace.ev[i], g_trace.ev[i + 1]);
+    if (e != cudaSuccess) return fail(ET_ERR_CUDA, "et_trace_get: %s", cudaGetErrorString(e));
+  }
+  return ET_OK;
+}
+
+int64_t et_launch_count(void) { return g_launches; }
 
 et_status et_prune_pack_query(int32_t rows, int32_t cols, et_dtype dtype, et_pattern pattern, double ratio,
                               int32_t tile_r, int32_t tile_c, int32_t group_rows, const uint32_t* host_mask_in,

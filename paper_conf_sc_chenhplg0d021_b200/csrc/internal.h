@@ -126,4 +126,9 @@ struct VPrep {
 };
 et_status vprep_run(const VPrep& v, cudaStream_t stream);
 
+// ---------------------------------------------------------------- tracing (api.cu)
+// Record a mark of `kind` on `stream` if tracing is enabled; counts one kernel launch.
+void trace_mark(int kind, cudaStream_t stream);
+void count_launch();
+
 }  // namespace et

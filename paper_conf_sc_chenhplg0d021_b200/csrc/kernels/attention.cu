@@ -417,6 +417,7 @@ et_status launch(const CUtensorMap& tm, const AParams& prm, dim3 grid, cudaStrea
   std::call_once(once, [&] { attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); });
   ET_CUDA(attr_err);
   kern<<<grid, kThreads, smem, stream>>>(tm, prm);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
 }

@@ -93,6 +93,7 @@ et_status cast_run(const void* src, et_dtype sdt, void* dst, et_dtype ddt, size_
   if (n == 0) return ET_OK;
   const size_t threads = 256, per = threads * 4;
   cast_kernel<<<(unsigned)((n + per - 1) / per), (unsigned)threads, 0, stream>>>(src, sdt, dst, ddt, n);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
 }
@@ -101,10 +102,12 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream) {
   if (v.wv->pattern != ET_PRUNE_ROW) return fail(ET_ERR_INTERNAL, "vprep: W_V is not row pruned");
   if (v.wo->pattern != ET_PRUNE_TILE) return fail(ET_ERR_UNSUPPORTED, "vprep: W_O must be tile pruned");
   vprep_heads_kernel<<<1, 32, 0, stream>>>(v.wv->idx, v.wv->nnz, v.heads, v.d_k, v.v_col, v.v_width);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   if (v.wv->rows_padded > 0) {
     vprep_bias_kernel<<<(v.wv->rows_padded + 255) / 256, 256, 0, stream>>>(v.wv->row_map, v.wv->rows_padded, v.bv,
                                                                            v.dtype, v.bv_packed);
+    count_launch();
     ET_CUDA(cudaGetLastError());
   }
   const int d = v.wo->rows;
@@ -112,6 +115,7 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream) {
                                                          v.wo->part_row_ptr, v.wo->tile_col, v.wo->rows / 16,
                                                          v.wo->kparts, v.wv->mask, v.bv, v.bo, v.dtype, d,
                                                          v.bo_folded);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
 }

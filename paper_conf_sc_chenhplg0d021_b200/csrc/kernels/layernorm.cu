@@ -125,6 +125,7 @@ et_status layernorm_run(const LnArgs& a, cudaStream_t stream) {
   const int threads = 256;
   const int blocks = (a.M * 32 + threads - 1) / threads;
   layernorm_kernel<<<blocks, threads, 0, stream>>>(a);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
 }

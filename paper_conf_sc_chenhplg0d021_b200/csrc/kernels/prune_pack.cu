@@ -267,25 +267,31 @@ et_status prune_pack_run(const PruneArgs& a, et_packed_weight* out, void* ws, si
     case ET_FP16:
       scores_kernel<__half><<<nb, tb, 0, stream>>>(static_cast<const __half*>(a.W), a.rows, a.cols, a.pattern,
                                                    a.tile_r, a.tile_c, units, scores);
+  count_launch();
       break;
     case ET_BF16:
       scores_kernel<__nv_bfloat16><<<nb, tb, 0, stream>>>(static_cast<const __nv_bfloat16*>(a.W), a.rows, a.cols,
                                                           a.pattern, a.tile_r, a.tile_c, units, scores);
+  count_launch();
       break;
     default:
       scores_kernel<float><<<nb, tb, 0, stream>>>(static_cast<const float*>(a.W), a.rows, a.cols, a.pattern,
                                                   a.tile_r, a.tile_c, units, scores);
+  count_launch();
   }
   ET_CUDA(cudaGetLastError());
   rank_kernel<<<nb, tb, 0, stream>>>(scores, units, a.n_prune, a.mask_in, keep);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   if (out->mask) {
     const int words = (units + 31) / 32;
     bitmap_kernel<<<(words + 127) / 128, 128, 0, stream>>>(keep, units, out->mask);
+  count_launch();
     ET_CUDA(cudaGetLastError());
   }
   index_kernel<<<1, 32, 0, stream>>>(keep, a.rows, a.cols, a.pattern, a.tile_r, a.tile_c, a.group_rows, out->idx,
                                      out->row_ptr, out->tile_col, out->row_map, out->part_row_ptr, counts);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   const bool pack_values = out->values != nullptr && a.dtype != ET_FP32 && a.tile_r == 16 && a.tile_c == 16 &&
                            a.pattern != ET_PRUNE_COL;
@@ -301,6 +307,7 @@ et_status prune_pack_run(const PruneArgs& a, et_packed_weight* out, void* ws, si
     pack_values_kernel<<<blocks, threads, 0, stream>>>(static_cast<const uint16_t*>(a.W), a.cols, a.pattern,
                                                        out->part_row_ptr, out->tile_col, out->row_map, counts,
                                                        kparts, static_cast<uint8_t*>(out->values), a.rows);
+  count_launch();
     ET_CUDA(cudaGetLastError());
   }
   int32_t hc[3];
@@ -324,6 +331,7 @@ et_status unpack_run(const et_packed_weight* w, void* dense, cudaStream_t stream
                                                 w->part_row_ptr, w->tile_col, w->row_map, w->ntiles,
                                                 w->pattern == ET_PRUNE_TILE ? w->rows / 16 : w->rows_padded / 16,
                                                 w->kparts, static_cast<uint16_t*>(dense));
+  count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
 }

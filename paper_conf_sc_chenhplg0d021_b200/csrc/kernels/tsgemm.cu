@@ -321,6 +321,7 @@ et_status launch_typed(const CUtensorMap& tm, const Params& prm, dim3 grid, cuda
   });
   ET_CUDA(attr_err);
   kern<<<grid, kThreads, kSmemBytes, stream>>>(tm, prm);
+  count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
 }
