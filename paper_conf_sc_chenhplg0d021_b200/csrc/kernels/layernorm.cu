@@ -16,7 +16,6 @@
 namespace et {
 namespace {
 
-constexpr int kMaxChunks = 16;  // N <= 16 * 128 = 2048
 
 __device__ __forceinline__ float4 ld_act4(const void* p, et_dtype dt, size_t idx) {
   if (dt == ET_FP32) return *reinterpret_cast<const float4*>(static_cast<const float*>(p) + idx);
@@ -47,87 +46,112 @@ __device__ __forceinline__ void st_act4(void* p, et_dtype dt, size_t idx, float4
   *reinterpret_cast<uint2*>(static_cast<uint16_t*>(p) + idx) = u;
 }
 
-__global__ void __launch_bounds__(256) layernorm_kernel(const LnArgs a) {
-  const int warp_g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+// One warp per row; NCH = ceil(N / 128) chunks of 4 columns per lane, NP split-K partial inputs.
+// All loads of the row are issued before any arithmetic so each warp has NCH * (NP + 2) 16/8-byte
+// requests in flight (the kernel is latency-bound otherwise).
+template <int NCH, int NP>
+__global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
+  const int row_i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
-  if (warp_g >= a.M) return;
-  const int nch = (a.N + 127) / 128;
-  const size_t row = (size_t)warp_g * a.N;
-  float4 v[kMaxChunks];
+  if (row_i >= a.M) return;
+  const size_t row = (size_t)row_i * a.N;
+  float4 part[NP][NCH];
+  float4 bias[NCH], res[NCH];
+  bool ok[NCH];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) ok[c] = c * 128 + lane * 4 < a.N;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int col = c * 128 + lane * 4;
+#pragma unroll
+    for (int q = 0; q < NP; ++q)
+      part[q][c] = ok[c] ? __ldcs(reinterpret_cast<const float4*>(a.part + (size_t)q * a.M * a.N + row + col))
+                         : make_float4(0.f, 0.f, 0.f, 0.f);
+    bias[c] = (ok[c] && a.bias) ? ld_act4(a.bias, a.dtype, col) : make_float4(0.f, 0.f, 0.f, 0.f);
+    res[c] = (ok[c] && a.resid) ? ld_act4(a.resid, a.resid_dtype, row + col) : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  float4 v[NCH];
   float s = 0.f;
 #pragma unroll
-  for (int c = 0; c < kMaxChunks; ++c) {
-    v[c] = make_float4(0.f, 0.f, 0.f, 0.f);
-    if (c < nch && c * 128 + lane * 4 < a.N) {
-      const int col = c * 128 + lane * 4;
-      float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-      for (int pidx = 0; pidx < a.nparts; ++pidx) {
-        const float4 t = *reinterpret_cast<const float4*>(a.part + (size_t)pidx * a.M * a.N + row + col);
-        x.x += t.x; x.y += t.y; x.z += t.z; x.w += t.w;
-      }
-      if (a.bias) {
-        const float4 b = ld_act4(a.bias, a.dtype, col);
-        x.x += b.x; x.y += b.y; x.z += b.z; x.w += b.w;
-      }
-      if (a.resid) {
-        const float4 r = ld_act4(a.resid, a.resid_dtype, row + col);
-        x.x += r.x; x.y += r.y; x.z += r.z; x.w += r.w;
-      }
-      v[c] = x;
-      s += x.x + x.y + x.z + x.w;
+  for (int c = 0; c < NCH; ++c) {
+    float4 x = part[0][c];
+#pragma unroll
+    for (int q = 1; q < NP; ++q) {
+      x.x += part[q][c].x; x.y += part[q][c].y; x.z += part[q][c].z; x.w += part[q][c].w;
     }
+    x.x += bias[c].x + res[c].x; x.y += bias[c].y + res[c].y;
+    x.z += bias[c].z + res[c].z; x.w += bias[c].w + res[c].w;
+    v[c] = x;
+    s += x.x + x.y + x.z + x.w;
   }
   if (a.gamma == nullptr) {   // no normalisation: out = sum(part) + bias (+ resid)
 #pragma unroll
-    for (int c = 0; c < kMaxChunks; ++c) {
-      if (c < nch && c * 128 + lane * 4 < a.N) {
-        const int col = c * 128 + lane * 4;
-        if (a.out_act) st_act4(a.out_act, a.dtype, row + col, v[c]);
-        if (a.out_resid) st_act4(a.out_resid, a.resid_dtype, row + col, v[c]);
-      }
+    for (int c = 0; c < NCH; ++c) {
+      if (!ok[c]) continue;
+      const int col = c * 128 + lane * 4;
+      if (a.out_act) st_act4(a.out_act, a.dtype, row + col, v[c]);
+      if (a.out_resid) st_act4(a.out_resid, a.resid_dtype, row + col, v[c]);
     }
     return;
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   const float mean = s / a.N;
-  float q = 0.f;
+  float q2 = 0.f;
 #pragma unroll
-  for (int c = 0; c < kMaxChunks; ++c) {
-    if (c < nch && c * 128 + lane * 4 < a.N) {
-      const float dx = v[c].x - mean, dy = v[c].y - mean, dz = v[c].z - mean, dw = v[c].w - mean;
-      q += dx * dx + dy * dy + dz * dz + dw * dw;
-    }
+  for (int c = 0; c < NCH; ++c) {
+    if (!ok[c]) continue;
+    const float dx = v[c].x - mean, dy = v[c].y - mean, dz = v[c].z - mean, dw = v[c].w - mean;
+    q2 += dx * dx + dy * dy + dz * dz + dw * dw;
   }
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
-  const float rstd = rsqrtf(q / a.N + a.eps);
+  for (int o = 16; o > 0; o >>= 1) q2 += __shfl_xor_sync(0xffffffffu, q2, o);
+  const float rstd = rsqrtf(q2 / a.N + a.eps);
 #pragma unroll
-  for (int c = 0; c < kMaxChunks; ++c) {
-    if (c < nch && c * 128 + lane * 4 < a.N) {
-      const int col = c * 128 + lane * 4;
-      const float4 gm = *reinterpret_cast<const float4*>(a.gamma + col);
-      const float4 bt = *reinterpret_cast<const float4*>(a.beta + col);
-      const float4 y = make_float4((v[c].x - mean) * rstd * gm.x + bt.x, (v[c].y - mean) * rstd * gm.y + bt.y,
-                                   (v[c].z - mean) * rstd * gm.z + bt.z, (v[c].w - mean) * rstd * gm.w + bt.w);
-      if (a.out_act) st_act4(a.out_act, a.dtype, row + col, y);
-      if (a.out_resid) st_act4(a.out_resid, a.resid_dtype, row + col, y);
-    }
+  for (int c = 0; c < NCH; ++c) {
+    if (!ok[c]) continue;
+    const int col = c * 128 + lane * 4;
+    const float4 gm = __ldg(reinterpret_cast<const float4*>(a.gamma + col));
+    const float4 bt = __ldg(reinterpret_cast<const float4*>(a.beta + col));
+    const float4 y = make_float4((v[c].x - mean) * rstd * gm.x + bt.x, (v[c].y - mean) * rstd * gm.y + bt.y,
+                                 (v[c].z - mean) * rstd * gm.z + bt.z, (v[c].w - mean) * rstd * gm.w + bt.w);
+    if (a.out_act) st_act4(a.out_act, a.dtype, row + col, y);
+    if (a.out_resid) st_act4(a.out_resid, a.resid_dtype, row + col, y);
   }
+}
+
+template <int NCH>
+et_status launch_np(const LnArgs& a, cudaStream_t stream) {
+  const int threads = 128;
+  const int blocks = (a.M * 32 + threads - 1) / threads;
+  switch (a.nparts) {
+    case 1: layernorm_kernel<NCH, 1><<<blocks, threads, 0, stream>>>(a); break;
+    case 2: layernorm_kernel<NCH, 2><<<blocks, threads, 0, stream>>>(a); break;
+    case 3: layernorm_kernel<NCH, 3><<<blocks, threads, 0, stream>>>(a); break;
+    case 4: layernorm_kernel<NCH, 4><<<blocks, threads, 0, stream>>>(a); break;
+    default: return fail(ET_ERR_UNSUPPORTED, "LayerNorm: up to 4 partial inputs (got %d)", a.nparts);
+  }
+  count_launch();
+  ET_CUDA(cudaGetLastError());
+  return ET_OK;
 }
 
 }  // namespace
 
 et_status layernorm_run(const LnArgs& a, cudaStream_t stream) {
-  if (a.N % 4 || a.N > 128 * kMaxChunks)
-    return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 4 and <= 2048 (got %d)", a.N);
+  if (a.N % 4 || a.N > 128 * 8)
+    return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 4 and <= 1024 (got %d)", a.N);
   if (a.M <= 0) return ET_OK;
-  const int threads = 256;
-  const int blocks = (a.M * 32 + threads - 1) / threads;
-  layernorm_kernel<<<blocks, threads, 0, stream>>>(a);
-  count_launch();
-  ET_CUDA(cudaGetLastError());
-  return ET_OK;
+  switch ((a.N + 127) / 128) {
+    case 1: return launch_np<1>(a, stream);
+    case 2: return launch_np<2>(a, stream);
+    case 3: return launch_np<3>(a, stream);
+    case 4: return launch_np<4>(a, stream);
+    case 5: return launch_np<5>(a, stream);
+    case 6: return launch_np<6>(a, stream);
+    case 7: return launch_np<7>(a, stream);
+    default: return launch_np<8>(a, stream);
+  }
 }
 
 }  // namespace et

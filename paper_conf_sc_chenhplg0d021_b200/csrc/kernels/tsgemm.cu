@@ -38,7 +38,11 @@ constexpr int kChunkTiles = 32;  // tiles per stage (16 KB)
 constexpr int kMaxKChunks = 12;  // K <= 768 per part
 constexpr int kMaxBChunks = 192; // tile chunks per CTA (one single-use full barrier each)
 constexpr int kAccCol = 384;     // first accumulator column (A uses [0, Kp/2) <= 384)
-constexpr int kThreads = 320;
+constexpr int kMmaWarps = 8;     // warps 0-7: MMA issue, one accumulator (16 TMEM columns) each
+// warps 8-15: epilogue, two groups of 4 (one per TMEM lane quarter)
+constexpr int kWarpA = 16;       // A producer (TMA + tcgen05.cp)
+constexpr int kWarpB = 17;       // tile producer + TMEM owner
+constexpr int kThreads = 18 * 32;
 
 struct SegDev {
   const int32_t* prp;       // part_row_ptr [kparts][tile_rows + 1]
@@ -67,21 +71,42 @@ struct Params {
 };
 
 struct __align__(8) Barriers {
-  uint64_t xfull[kNXS], xempty[kNXS], afill[kMaxKChunks], accf[8], bfull[kMaxBChunks];
+  uint64_t xfull[kNXS], xempty[kNXS], afill[kMaxKChunks];
+  uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
+  uint64_t bfull[kMaxBChunks];
   uint32_t tmem_base;
-  int quads_done[2];   // per warpgroup, written by its leader thread after each quad
+  int rows_seen[2];   // per epilogue group: rows whose MMAs were observed complete (in row order)
 };
 
 constexpr size_t kSmemX = (size_t)kNXS * 16384;
 constexpr size_t kSmemB = (size_t)kNBS * kChunkTiles * 512;
 constexpr size_t kSmemBytes = 1024 + kSmemX + kSmemB + sizeof(Barriers);
 
+// GELU(x) = 0.5 x (1 + erf(x / sqrt 2)) (reading C-12)
 __device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * (1.0f + erff(x * 0.70710678118654752f)); }
 
+template <bool kBF16>
+__device__ __forceinline__ void load_bias16(const void* bias, int col, float (&b)[16]) {
+  if (bias == nullptr) {
+#pragma unroll
+    for (int c = 0; c < 16; ++c) b[c] = 0.f;
+    return;
+  }
+  const uint4* p = reinterpret_cast<const uint4*>(static_cast<const uint16_t*>(bias) + col);
+  const uint4 u0 = __ldg(p), u1 = __ldg(p + 1);
+  const uint32_t w[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    const float2 f = unpack2<kBF16>(w[c]);
+    b[2 * c] = f.x;
+    b[2 * c + 1] = f.y;
+  }
+}
+
+// epilogue of one 16-feature group of one token row
 template <int kEpi, bool kBF16>
 __device__ __forceinline__ void epilogue_store(const Params& p, const SegDev& sg, int row_g, int col_local,
                                                const float (&acc)[16], int z) {
-  // col_local: first output feature of this 16-wide group within the segment
   using T = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
   if constexpr (kEpi == ET_EPI_F32) {
     float* Y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row_g * p.ldy + sg.out_col + col_local;
@@ -89,15 +114,12 @@ __device__ __forceinline__ void epilogue_store(const Params& p, const SegDev& sg
     for (int c = 0; c < 16; c += 4)
       *reinterpret_cast<float4*>(Y + c) = make_float4(acc[c], acc[c + 1], acc[c + 2], acc[c + 3]);
   } else {
+    float b[16];
+    load_bias16<kBF16>(sg.bias, col_local, b);
     float v[16];
-    const T* b = static_cast<const T*>(sg.bias);
 #pragma unroll
     for (int c = 0; c < 16; ++c) {
-      float x = acc[c];
-      if (b) {
-        if constexpr (kBF16) x += __bfloat162float(b[col_local + c]);
-        else x += __half2float(b[col_local + c]);
-      }
+      float x = acc[c] + b[c];
       if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
         if (sg.apply_scale) x *= sg.scale;
       } else if constexpr (kEpi == ET_EPI_BIAS_GELU) {
@@ -136,7 +158,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int pb = rp[pc.i0], pe = rp[pc.i1];    // this CTA's packed tiles [pb, pe)
   const int nchunks = (pe - pb + kChunkTiles - 1) / kChunkTiles;
   const int nrows = pc.i1 - pc.i0;
-  const int nquads = (nrows + 3) / 4;
+  const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
 
   if (nchunks > kMaxBChunks) __trap();   // host sizes pieces so this cannot happen
   if (threadIdx.x == 0) {
@@ -145,21 +167,24 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       mbar_init(&bar.xempty[i], 1);
     }
     for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.afill[i], 1);
+    for (int i = 0; i < kMmaWarps; ++i) {
+      mbar_init(&bar.acc_full[i], 1);
+      mbar_init(&bar.acc_empty[i], 4);
+    }
     // one full barrier per tile chunk, each completing exactly once (parity 0): a warp may skip
     // ahead to a chunk whose ring slot has not even received its previous fill, and a parity wait
     // on a reused barrier cannot tell those phases apart.
     for (int i = 0; i < nchunks; ++i) mbar_init(&bar.bfull[i], 1);
-    bar.quads_done[0] = bar.quads_done[1] = 0;
-    for (int i = 0; i < 8; ++i) mbar_init(&bar.accf[i], 1);
+    bar.rows_seen[0] = bar.rows_seen[1] = 0;
     fence_mbar_init();
   }
-  if (warp == 9) tmem_alloc<512>(&bar.tmem_base);
+  if (warp == kWarpB) tmem_alloc<512>(&bar.tmem_base);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = bar.tmem_base;
 
-  if (warp == 8) {
+  if (warp == kWarpA) {
     // ===================== A producer: X block -> smem (TMA) -> TMEM (tcgen05.cp)
     if (lane == 0) {
       tma_prefetch_desc(&tmap_x);
@@ -188,97 +213,100 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         }
       }
     }
-  } else if (warp == 9) {
+  } else if (warp == kWarpB) {
     // ===================== tile producer: packed tiles -> smem ring (bulk copies)
-    // Slot reuse is quad-granular: chunk c may overwrite chunk c - kNBS once every quad (4 tile
-    // rows) touching chunk c - kNBS has completed its MMAs.  Warpgroup g owns quads g, g+2, ...
-    // and bumps quads_done[g] after each quad's epilogue barrier (its MMAs are complete then).
+    // Slot reuse is row-granular: chunk c may overwrite chunk c - kNBS once every tile row touching
+    // chunk c - kNBS has completed its MMAs.  Epilogue group g owns rows 8k + 4g + a (a < 4) and
+    // publishes rows_seen[g] in that order.  (A single row spans at most 3 chunks < kNBS, so the
+    // producer never waits for a row that itself needs the chunk being loaded.)
     if (lane == 0) {
       const uint8_t* vals = sg.values + (size_t)pb * 512;
-      int qq = 0;             // last quad that starts before the end of the chunk being recycled
+      int tl = 0;   // last local row that starts before the end of the chunk being recycled
       for (int c = 0; c < nchunks; ++c) {
         const int slot = c % kNBS;
         if (c >= kNBS) {
-          const int cr = c - kNBS;
-          const int end_tile = pb + (cr + 1) * kChunkTiles;   // tiles of chunk cr are < end_tile
-          while (qq + 1 < nquads && rp[min(pc.i0 + (qq + 1) * 4, pc.i1)] < end_tile) ++qq;
-          const int need0 = qq / 2 + 1, need1 = (qq + 1) / 2;   // quads 0,2,.. / 1,3,.. up to qq
-          while (ld_acquire_shared(&bar.quads_done[0]) < need0) {}
-          while (ld_acquire_shared(&bar.quads_done[1]) < need1) {}
+          const int end_tile = pb + (c - kNBS + 1) * kChunkTiles;
+          while (tl + 1 < nrows && rp[pc.i0 + tl + 1] < end_tile) ++tl;
+          const int full = (tl + 1) / kMmaWarps, rem = (tl + 1) % kMmaWarps;
+          const int need0 = 4 * full + min(max(rem, 0), 4);
+          const int need1 = 4 * full + min(max(rem - 4, 0), 4);
+          while (ld_acquire_shared(&bar.rows_seen[0]) < need0) {}
+          while (ld_acquire_shared(&bar.rows_seen[1]) < need1) {}
         }
         const int nt = min(kChunkTiles, pe - pb - c * kChunkTiles);
         mbar_expect_tx(&bar.bfull[c], nt * 512);
         bulk_load(sB + slot * (kChunkTiles * 512), vals + (size_t)c * kChunkTiles * 512, nt * 512, &bar.bfull[c]);
       }
     }
-  } else {
-    // ===================== MMA + epilogue warps (2 warpgroups x 4 warps)
-    const int g = warp >> 2, jw = warp & 3;
+  } else if (warp < kMmaWarps) {
+    // ===================== MMA warps: warp w issues the chains of tile rows w, w+8, w+16, ...
     const uint32_t idesc = make_idesc_f16(128, 16, kBF16 ? 1 : 0, 0, 0);
     const uint32_t d_tmem = tbase + kAccCol + warp * 16;
     const uint32_t sB_u32 = smem_u32(sB);
     const int kbase = z * 48;   // first tile column of this K part
     int a_ready = -1;           // highest A chunk known filled
     int cur_chunk = -1;         // B chunk whose full barrier was last waited
-    int round = 0;
-    for (int q = g; q < nquads; q += 2, ++round) {
-      const int t = q * 4 + jw;                 // local tile row of this warp in this round
-      if (t < nrows) {
-        const int i = pc.i0 + t;
-        const int p0 = rp[i], p1 = rp[i + 1];
-        for (int base = p0; base < p1; base += 32) {
-          const int mycol = (base + lane < p1) ? sg.tile_col[base + lane] : 0;
-          const int n = min(32, p1 - base);
-          for (int u = 0; u < n; ++u) {
-            const int pp = base + u;
-            const int kc = __shfl_sync(0xffffffffu, mycol, u) - kbase;
-            const int c = (pp - pb) / kChunkTiles;
-            if (c != cur_chunk) {
-              mbar_wait_warp(&bar.bfull[c], 0);
-              cur_chunk = c;
-              tc_fence_after();
-            }
-            const int ach = kc >> 2;
-            if (ach > a_ready) {
-              mbar_wait_warp(&bar.afill[ach], 0);
-              a_ready = ach;
-              tc_fence_after();
-            }
-            const uint32_t baddr = sB_u32 + (c % kNBS) * (kChunkTiles * 512) + ((pp - pb) % kChunkTiles) * 512;
-            mma_ts_warp(d_tmem, tbase + kc * 8, make_sdesc(baddr, 128, 256, kLayoutNone), idesc, pp != p0);
+    for (int k = 0; k < nrounds; ++k) {
+      const int t = k * kMmaWarps + warp;
+      if (t >= nrows) break;
+      if (k > 0) {   // the epilogue group must have read this accumulator's previous row
+        mbar_wait_warp(&bar.acc_empty[warp], (k - 1) & 1);
+        tc_fence_after();
+      }
+      const int i = pc.i0 + t;
+      const int p0 = rp[i], p1 = rp[i + 1];
+      for (int base = p0; base < p1; base += 32) {
+        const int mycol = (base + lane < p1) ? sg.tile_col[base + lane] : 0;
+        const int n = min(32, p1 - base);
+        for (int u = 0; u < n; ++u) {
+          const int pp = base + u;
+          const int kc = __shfl_sync(0xffffffffu, mycol, u) - kbase;
+          const int c = (pp - pb) / kChunkTiles;
+          if (c != cur_chunk) {
+            mbar_wait_warp(&bar.bfull[c], 0);
+            cur_chunk = c;
+            tc_fence_after();
           }
+          const int ach = kc >> 2;
+          if (ach > a_ready) {
+            mbar_wait_warp(&bar.afill[ach], 0);
+            a_ready = ach;
+            tc_fence_after();
+          }
+          const uint32_t baddr = sB_u32 + (c % kNBS) * (kChunkTiles * 512) + ((pp - pb) % kChunkTiles) * 512;
+          mma_ts_warp(d_tmem, tbase + kc * 8, make_sdesc(baddr, 128, 256, kLayoutNone), idesc, pp != p0);
         }
       }
-      mma_commit_warp(&bar.accf[warp]);
-
-      // ---- epilogue of quad q: this warp reads lane quarter jw of the 4 accumulators of its group
-      float acc[4][16];
-#pragma unroll
-      for (int a = 0; a < 4; ++a) mbar_wait_warp(&bar.accf[g * 4 + a], round & 1);
-      tc_fence_after();
-#pragma unroll
+      mma_commit_warp(&bar.acc_full[warp]);   // fires when this row's MMAs are complete
+    }
+  } else {
+    // ===================== epilogue warps: group g drains the accumulators of MMA warps 4g..4g+3
+    const int e = warp - kMmaWarps;
+    const int g = e >> 2;
+    const int quarter = warp & 3;               // TMEM lane quarter this warp may access
+    const int row_g = m0 + quarter * 32 + lane;
+    int seen = 0;
+    for (int k = 0; k < nrounds; ++k) {
+#pragma unroll 1
       for (int a = 0; a < 4; ++a) {
+        const int w = g * 4 + a;
+        const int t = k * kMmaWarps + w;
+        if (t >= nrows) break;
+        mbar_wait_warp(&bar.acc_full[w], k & 1);
+        tc_fence_after();
+        if (quarter == 0 && lane == 0) st_release_shared(&bar.rows_seen[g], ++seen);   // row's B tiles free
         uint32_t r[16];
-        tmem_ld16(tbase + kAccCol + (g * 4 + a) * 16 + ((uint32_t)(jw * 32) << 16), r);
+        tmem_ld16(tbase + kAccCol + w * 16 + ((uint32_t)(quarter * 32) << 16), r);
         tmem_ld_wait();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&bar.acc_empty[w]);   // accumulator may take its next row
+        const int i = pc.i0 + t;
+        float acc[16];
+        const bool empty_row = rp[i + 1] == rp[i];      // fully pruned tile row: never written
 #pragma unroll
-        for (int c = 0; c < 16; ++c) acc[a][c] = __uint_as_float(r[c]);
-      }
-      tc_fence_before();
-      named_bar_sync(1 + g, 128);
-      __syncwarp();
-      if (jw == 0 && lane == 0) st_release_shared(&bar.quads_done[g], round + 1);   // quad's MMAs complete
-      const int row_g = m0 + jw * 32 + lane;
-#pragma unroll
-      for (int a = 0; a < 4; ++a) {
-        const int ta = q * 4 + a;
-        if (ta >= nrows) continue;
-        const int i = pc.i0 + ta;
-        if (rp[i + 1] == rp[i]) {   // fully pruned tile row: the accumulator was never written
-#pragma unroll
-          for (int c = 0; c < 16; ++c) acc[a][c] = 0.0f;
-        }
-        if (row_g < p.M) epilogue_store<kEpi, kBF16>(p, sg, row_g, i * 16, acc[a], z);
+        for (int c = 0; c < 16; ++c) acc[c] = empty_row ? 0.f : __uint_as_float(r[c]);
+        if (row_g < p.M) epilogue_store<kEpi, kBF16>(p, sg, row_g, i * 16, acc, z);
       }
     }
   }
@@ -286,7 +314,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   __syncwarp();   // producer warps: lane 0 ran the loops alone; reconverge before the block barrier
   tc_fence_before();
   __syncthreads();
-  if (warp == 9) {
+  if (warp == kWarpB) {
     __syncwarp();
     tc_fence_after();
     tmem_dealloc<512>(tbase);   // .sync.aligned: the whole warp, converged
@@ -369,9 +397,10 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   const int mblocks = (a.M + 127) / 128;
   int total_rows = 0;
   for (int s = 0; s < a.nseg; ++s) total_rows += a.seg[s].tile_rows;
-  // pieces: aim for ~1-2 waves of CTAs over 148 SMs, >= 8 tile rows per piece
+  // pieces: one wave of CTAs over the 148 SMs (a nearly empty second wave would double the time)
   const int target_ctas = 148;
-  int pieces_total = (target_ctas + mblocks * kparts - 1) / (mblocks * kparts);
+  int pieces_total = target_ctas / (mblocks * kparts);
+  if (pieces_total < 1) pieces_total = 1;
   if (pieces_total < a.nseg) pieces_total = a.nseg;
   int np = 0;
   for (int s = 0; s < a.nseg; ++s) {
