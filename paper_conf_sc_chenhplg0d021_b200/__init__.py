@@ -373,4 +373,6 @@ _sig("et_trace_begin", ctypes.c_int, [_i32])
 _sig("et_trace_end", ctypes.c_int, [ctypes.POINTER(_i32)])
 _sig("et_trace_get", ctypes.c_int, [_i32, ctypes.POINTER(_i32), ctypes.POINTER(_f32)])
 _sig("et_launch_count", ctypes.c_int64, [])
+if hasattr(_lib, "et_diag_gemm_timeline"):
+    _sig("et_diag_gemm_timeline", ctypes.c_int, [_vp])
 SYMBOLS += ["et_trace_begin", "et_trace_end", "et_trace_get", "et_launch_count"]

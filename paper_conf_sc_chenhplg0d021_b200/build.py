@@ -51,7 +51,7 @@ def build(verbose: bool = False, force: bool = False, debug: bool = False) -> st
     nvcc = _nvcc()
     bdir = BUILD + ("_dbg" if debug else "")
     lib = os.path.join(bdir, "libet_dbg.so") if debug else LIB
-    flags = FLAGS + (["-DET_WATCHDOG"] if debug else [])
+    flags = FLAGS + (["-DET_WATCHDOG", "-DET_TIMELINE"] if debug else [])
     os.makedirs(bdir, exist_ok=True)
     hdr_mtime = max([os.path.getmtime(h) for h in _headers()] + [0.0])
     jobs = []

@@ -150,7 +150,7 @@ et_status et_prune_pack_query(int32_t rows, int32_t cols, et_dtype dtype, et_pat
   if (mask_bytes) *mask_bytes = (size_t)((units + 31) / 32) * 4;
   if (idx_bytes) *idx_bytes = (size_t)(units > 0 ? units : 1) * 4;
   if (rowptr_bytes) *rowptr_bytes = (size_t)(tile_rows_max + 1) * 4;
-  if (tilecol_bytes) *tilecol_bytes = (size_t)(tiles_max > 0 ? tiles_max : 1) * 4;
+  if (tilecol_bytes) *tilecol_bytes = (size_t)(tiles_max > 0 ? tiles_max : 1) * 4 + 16;   // +16: aligned bulk reads
   if (rowmap_bytes) *rowmap_bytes = pattern == ET_PRUNE_ROW ? (size_t)tile_rows_max * 16 * 4 : 4;
   if (partrowptr_bytes) *partrowptr_bytes = (size_t)kparts * (tile_rows_max + 1) * 4;
   const bool has_values = tile_r == 16 && tile_c == 16 && dtype != ET_FP32 && pattern != ET_PRUNE_COL &&

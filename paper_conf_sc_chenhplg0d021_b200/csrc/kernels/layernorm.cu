@@ -17,11 +17,13 @@ namespace et {
 namespace {
 
 
-__device__ __forceinline__ float4 ld_act4(const void* p, et_dtype dt, size_t idx) {
-  if (dt == ET_FP32) return *reinterpret_cast<const float4*>(static_cast<const float*>(p) + idx);
+template <int DT>
+__device__ __forceinline__ float4 ld_act4(const void* p, size_t idx) {
+  constexpr et_dtype dt = (et_dtype)DT;
+  if constexpr (dt == ET_FP32) return *reinterpret_cast<const float4*>(static_cast<const float*>(p) + idx);
   const uint2 u = *reinterpret_cast<const uint2*>(static_cast<const uint16_t*>(p) + idx);
   float2 a, b;
-  if (dt == ET_BF16) {
+  if constexpr (dt == ET_BF16) {
     a = unpack2<true>(u.x);
     b = unpack2<true>(u.y);
   } else {
@@ -30,13 +32,15 @@ __device__ __forceinline__ float4 ld_act4(const void* p, et_dtype dt, size_t idx
   }
   return make_float4(a.x, a.y, b.x, b.y);
 }
-__device__ __forceinline__ void st_act4(void* p, et_dtype dt, size_t idx, float4 v) {
-  if (dt == ET_FP32) {
+template <int DT>
+__device__ __forceinline__ void st_act4(void* p, size_t idx, float4 v) {
+  constexpr et_dtype dt = (et_dtype)DT;
+  if constexpr (dt == ET_FP32) {
     *reinterpret_cast<float4*>(static_cast<float*>(p) + idx) = v;
     return;
   }
   uint2 u;
-  if (dt == ET_BF16) {
+  if constexpr (dt == ET_BF16) {
     u.x = pack2<true>(v.x, v.y);
     u.y = pack2<true>(v.z, v.w);
   } else {
@@ -49,7 +53,7 @@ __device__ __forceinline__ void st_act4(void* p, et_dtype dt, size_t idx, float4
 // One warp per row; NCH = ceil(N / 128) chunks of 4 columns per lane, NP split-K partial inputs.
 // All loads of the row are issued before any arithmetic so each warp has NCH * (NP + 2) 16/8-byte
 // requests in flight (the kernel is latency-bound otherwise).
-template <int NCH, int NP>
+template <int NCH, int NP, int DT, int RT>
 __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
   const int row_i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
@@ -67,8 +71,8 @@ __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
     for (int q = 0; q < NP; ++q)
       part[q][c] = ok[c] ? __ldcs(reinterpret_cast<const float4*>(a.part + (size_t)q * a.M * a.N + row + col))
                          : make_float4(0.f, 0.f, 0.f, 0.f);
-    bias[c] = (ok[c] && a.bias) ? ld_act4(a.bias, a.dtype, col) : make_float4(0.f, 0.f, 0.f, 0.f);
-    res[c] = (ok[c] && a.resid) ? ld_act4(a.resid, a.resid_dtype, row + col) : make_float4(0.f, 0.f, 0.f, 0.f);
+    bias[c] = (ok[c] && a.bias) ? ld_act4<DT>(a.bias, col) : make_float4(0.f, 0.f, 0.f, 0.f);
+    res[c] = (ok[c] && a.resid) ? ld_act4<RT>(a.resid, row + col) : make_float4(0.f, 0.f, 0.f, 0.f);
   }
   float4 v[NCH];
   float s = 0.f;
@@ -89,8 +93,8 @@ __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
     for (int c = 0; c < NCH; ++c) {
       if (!ok[c]) continue;
       const int col = c * 128 + lane * 4;
-      if (a.out_act) st_act4(a.out_act, a.dtype, row + col, v[c]);
-      if (a.out_resid) st_act4(a.out_resid, a.resid_dtype, row + col, v[c]);
+      if (a.out_act) st_act4<DT>(a.out_act, row + col, v[c]);
+      if (a.out_resid) st_act4<RT>(a.out_resid, row + col, v[c]);
     }
     return;
   }
@@ -115,25 +119,35 @@ __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
     const float4 bt = __ldg(reinterpret_cast<const float4*>(a.beta + col));
     const float4 y = make_float4((v[c].x - mean) * rstd * gm.x + bt.x, (v[c].y - mean) * rstd * gm.y + bt.y,
                                  (v[c].z - mean) * rstd * gm.z + bt.z, (v[c].w - mean) * rstd * gm.w + bt.w);
-    if (a.out_act) st_act4(a.out_act, a.dtype, row + col, y);
-    if (a.out_resid) st_act4(a.out_resid, a.resid_dtype, row + col, y);
+    if (a.out_act) st_act4<DT>(a.out_act, row + col, y);
+    if (a.out_resid) st_act4<RT>(a.out_resid, row + col, y);
   }
 }
 
-template <int NCH>
+template <int NCH, int DT, int RT>
 et_status launch_np(const LnArgs& a, cudaStream_t stream) {
   const int threads = 128;
   const int blocks = (a.M * 32 + threads - 1) / threads;
   switch (a.nparts) {
-    case 1: layernorm_kernel<NCH, 1><<<blocks, threads, 0, stream>>>(a); break;
-    case 2: layernorm_kernel<NCH, 2><<<blocks, threads, 0, stream>>>(a); break;
-    case 3: layernorm_kernel<NCH, 3><<<blocks, threads, 0, stream>>>(a); break;
-    case 4: layernorm_kernel<NCH, 4><<<blocks, threads, 0, stream>>>(a); break;
+    case 1: layernorm_kernel<NCH, 1, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
+    case 2: layernorm_kernel<NCH, 2, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
+    case 3: layernorm_kernel<NCH, 3, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
+    case 4: layernorm_kernel<NCH, 4, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
     default: return fail(ET_ERR_UNSUPPORTED, "LayerNorm: up to 4 partial inputs (got %d)", a.nparts);
   }
   count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
+}
+
+template <int NCH>
+et_status launch_dt(const LnArgs& a, cudaStream_t stream) {
+  const int dt = a.dtype, rt = a.resid ? a.resid_dtype : (a.out_resid ? a.resid_dtype : a.dtype);
+  if (dt == ET_FP16 && rt == ET_FP16) return launch_np<NCH, ET_FP16, ET_FP16>(a, stream);
+  if (dt == ET_FP16 && rt == ET_FP32) return launch_np<NCH, ET_FP16, ET_FP32>(a, stream);
+  if (dt == ET_BF16 && rt == ET_BF16) return launch_np<NCH, ET_BF16, ET_BF16>(a, stream);
+  if (dt == ET_BF16 && rt == ET_FP32) return launch_np<NCH, ET_BF16, ET_FP32>(a, stream);
+  return fail(ET_ERR_UNSUPPORTED, "LayerNorm: dtype pair (%d, %d) not supported", dt, rt);
 }
 
 }  // namespace
@@ -143,14 +157,14 @@ et_status layernorm_run(const LnArgs& a, cudaStream_t stream) {
     return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 4 and <= 1024 (got %d)", a.N);
   if (a.M <= 0) return ET_OK;
   switch ((a.N + 127) / 128) {
-    case 1: return launch_np<1>(a, stream);
-    case 2: return launch_np<2>(a, stream);
-    case 3: return launch_np<3>(a, stream);
-    case 4: return launch_np<4>(a, stream);
-    case 5: return launch_np<5>(a, stream);
-    case 6: return launch_np<6>(a, stream);
-    case 7: return launch_np<7>(a, stream);
-    default: return launch_np<8>(a, stream);
+    case 1: return launch_dt<1>(a, stream);
+    case 2: return launch_dt<2>(a, stream);
+    case 3: return launch_dt<3>(a, stream);
+    case 4: return launch_dt<4>(a, stream);
+    case 5: return launch_dt<5>(a, stream);
+    case 6: return launch_dt<6>(a, stream);
+    case 7: return launch_dt<7>(a, stream);
+    default: return launch_dt<8>(a, stream);
   }
 }
 

@@ -24,25 +24,48 @@
 #include <cstdint>
 #include <mutex>
 #include <type_traits>
+#include <algorithm>
 
 #include "../internal.h"
 #include "../ptx.cuh"
 
 namespace et {
+
+#ifdef ET_TIMELINE
+// Debug builds only: %globaltimer stamps of CTA (0, 0, 0) of the most recent launch.
+//   slot 0: start; 1: metadata staged; 2..13: A chunk j copied to TMEM (producer); 14: last tile chunk
+//   issued; 16 + 8*w + 2*k, +1: MMA warp w, round k issue start / commit; 96 + 2*r, +1: epilogue row r
+//   accumulator observed / stores issued; 255: end.
+__device__ unsigned long long g_timeline[512];
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define ET_TL(slot)                                                              \
+  do {                                                                           \
+    if (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0 && (slot) < 512) g_timeline[(slot)] = gtime(); \
+  } while (0)
+#else
+#define ET_TL(slot) do {} while (0)
+#endif
+
 namespace {
 
 constexpr int kMaxPieces = 64;
-constexpr int kNXS = 4;          // X staging stages (16 KB each: 128 rows x 64 K)
+constexpr int kNXS = 3;          // X staging stages (16 KB each: 128 rows x 64 K)
 constexpr int kNBS = 8;          // tile staging stages
 constexpr int kChunkTiles = 32;  // tiles per stage (16 KB)
 constexpr int kMaxKChunks = 12;  // K <= 768 per part
 constexpr int kMaxBChunks = 192; // tile chunks per CTA (one single-use full barrier each)
+constexpr int kMaxRows = 256;    // tile rows per CTA (row pointers and bias staged in smem)
 constexpr int kAccCol = 384;     // first accumulator column (A uses [0, Kp/2) <= 384)
 constexpr int kMmaWarps = 8;     // warps 0-7: MMA issue, one accumulator (16 TMEM columns) each
 // warps 8-15: epilogue, two groups of 4 (one per TMEM lane quarter)
-constexpr int kWarpA = 16;       // A producer (TMA + tcgen05.cp)
+constexpr int kWarpA = 16;       // A producer: TMA of the X block into the smem ring
 constexpr int kWarpB = 17;       // tile producer + TMEM owner
-constexpr int kThreads = 18 * 32;
+constexpr int kWarpCp = 18;      // A producer: tcgen05.cp smem -> TMEM (runs behind the TMA thread)
+constexpr int kThreads = 19 * 32;
 
 struct SegDev {
   const int32_t* prp;       // part_row_ptr [kparts][tile_rows + 1]
@@ -74,78 +97,45 @@ struct __align__(8) Barriers {
   uint64_t xfull[kNXS], xempty[kNXS], afill[kMaxKChunks];
   uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
   uint64_t bfull[kMaxBChunks];
+  int tcol[kNBS][kChunkTiles + 4];   // tile columns of the staged tiles (from a 16-byte aligned start)
+  int rptr[kMaxRows + 1];        // this CTA's row pointers, relative to its first tile
+  uint32_t bias_s[kMaxRows * 8]; // this CTA's bias slice (16-bit pairs)
   uint32_t tmem_base;
   int rows_seen[2];   // per epilogue group: rows whose MMAs were observed complete (in row order)
 };
 
 constexpr size_t kSmemX = (size_t)kNXS * 16384;
 constexpr size_t kSmemB = (size_t)kNBS * kChunkTiles * 512;
-constexpr size_t kSmemBytes = 1024 + kSmemX + kSmemB + sizeof(Barriers);
+constexpr size_t kSmemStage = 8 * 4096;   // epilogue staging: 32 rows x 128 B per epilogue warp (SW128)
+constexpr size_t kSmemBytes = 1024 + kSmemX + kSmemB + kSmemStage + sizeof(Barriers);
 
-// GELU(x) = 0.5 x (1 + erf(x / sqrt 2)) (reading C-12)
-__device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * (1.0f + erff(x * 0.70710678118654752f)); }
-
-template <bool kBF16>
-__device__ __forceinline__ void load_bias16(const void* bias, int col, float (&b)[16]) {
-  if (bias == nullptr) {
-#pragma unroll
-    for (int c = 0; c < 16; ++c) b[c] = 0.f;
-    return;
-  }
-  const uint4* p = reinterpret_cast<const uint4*>(static_cast<const uint16_t*>(bias) + col);
-  const uint4 u0 = __ldg(p), u1 = __ldg(p + 1);
-  const uint32_t w[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
-#pragma unroll
-  for (int c = 0; c < 8; ++c) {
-    const float2 f = unpack2<kBF16>(w[c]);
-    b[2 * c] = f.x;
-    b[2 * c + 1] = f.y;
-  }
-}
-
-// epilogue of one 16-feature group of one token row
-template <int kEpi, bool kBF16>
-__device__ __forceinline__ void epilogue_store(const Params& p, const SegDev& sg, int row_g, int col_local,
-                                               const float (&acc)[16], int z) {
-  using T = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
-  if constexpr (kEpi == ET_EPI_F32) {
-    float* Y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row_g * p.ldy + sg.out_col + col_local;
-#pragma unroll
-    for (int c = 0; c < 16; c += 4)
-      *reinterpret_cast<float4*>(Y + c) = make_float4(acc[c], acc[c + 1], acc[c + 2], acc[c + 3]);
-  } else {
-    float b[16];
-    load_bias16<kBF16>(sg.bias, col_local, b);
-    float v[16];
-#pragma unroll
-    for (int c = 0; c < 16; ++c) {
-      float x = acc[c] + b[c];
-      if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
-        if (sg.apply_scale) x *= sg.scale;
-      } else if constexpr (kEpi == ET_EPI_BIAS_GELU) {
-        x = gelu_erf(x);
-      } else if constexpr (kEpi == ET_EPI_BIAS_RELU) {
-        x = fmaxf(x, 0.0f);
-      }
-      v[c] = x;
-    }
-    uint32_t packed[8];
-#pragma unroll
-    for (int c = 0; c < 8; ++c) packed[c] = pack2<kBF16>(v[2 * c], v[2 * c + 1]);
-    T* Y = static_cast<T*>(p.Y) + (size_t)row_g * p.ldy + sg.out_col + col_local;
-    *reinterpret_cast<uint4*>(Y) = make_uint4(packed[0], packed[1], packed[2], packed[3]);
-    *reinterpret_cast<uint4*>(Y + 8) = make_uint4(packed[4], packed[5], packed[6], packed[7]);
-  }
+// GELU(x) = x Phi(x) = 0.5 x (1 + erf(x / sqrt 2)) (reading C-12), evaluated as
+//   0.5 erfc(t) = 2^(-g(t) - 1),  t = |x| / sqrt 2 clamped to 4,  g(t) = -log2 erfc(t) ~ t q(t)
+// with q a degree-5 polynomial fitted on [0, 4] (tools/fit_gelu.py): |GELU error| <= 6.3e-7 in FP32
+// (below FP16/BF16 output resolution) for ~12 instructions and one ex2, half the cost of erff().
+__device__ __forceinline__ float gelu_erf(float x) {
+  const float t = fminf(fabsf(x) * 0.70710678118654752f, 4.0f);
+  float q = -0.00015888f;
+  q = fmaf(q, t, 0.0037465857f);
+  q = fmaf(q, t, -0.0310388145f);
+  q = fmaf(q, t, 0.1498060619f);
+  q = fmaf(q, t, 0.9181324485f);
+  q = fmaf(q, t, 1.6279282351f);
+  float e;   // 0.5 * erfc(t)
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e) : "f"(-fmaf(t, q, 1.0f)));
+  return x * (x >= 0.f ? 1.0f - e : e);
 }
 
 template <int kEpi, bool kBF16>
 __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
+                                                             const __grid_constant__ CUtensorMap tmap_y,
                                                              const __grid_constant__ Params p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sX = smem;
   uint8_t* sB = smem + kSmemX;
-  Barriers& bar = *reinterpret_cast<Barriers*>(smem + kSmemX + kSmemB);
+  uint8_t* sStage = smem + kSmemX + kSmemB;
+  Barriers& bar = *reinterpret_cast<Barriers*>(smem + kSmemX + kSmemB + kSmemStage);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -160,7 +150,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int nrows = pc.i1 - pc.i0;
   const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
 
-  if (nchunks > kMaxBChunks) __trap();   // host sizes pieces so this cannot happen
+  if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
+  if (threadIdx.x == 0) ET_TL(0);
   if (threadIdx.x == 0) {
     for (int i = 0; i < kNXS; ++i) {
       mbar_init(&bar.xfull[i], 1);
@@ -179,20 +170,34 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     fence_mbar_init();
   }
   if (warp == kWarpB) tmem_alloc<512>(&bar.tmem_base);
+  // stage the per-CTA metadata once (one global round trip instead of one per tile row)
+  for (int i = threadIdx.x; i <= nrows; i += blockDim.x) bar.rptr[i] = rp[pc.i0 + i] - pb;
+  if constexpr (kEpi != ET_EPI_F32) {
+    const uint32_t* bsrc = static_cast<const uint32_t*>(sg.bias);
+    for (int i = threadIdx.x; i < nrows * 8; i += blockDim.x)
+      bar.bias_s[i] = bsrc ? __ldg(bsrc + (size_t)pc.i0 * 8 + i) : 0u;
+  }
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = bar.tmem_base;
+  if (threadIdx.x == 0) ET_TL(1);
 
   if (warp == kWarpA) {
-    // ===================== A producer: X block -> smem (TMA) -> TMEM (tcgen05.cp)
+    // ===================== A producer (TMA): X block -> smem ring, up to kNXS chunks ahead
     if (lane == 0) {
       tma_prefetch_desc(&tmap_x);
       const int kx0 = z * p.Kp;
-      for (int j = 0; j < nk && j < kNXS; ++j) {
-        mbar_expect_tx(&bar.xfull[j], p.box_rows * 128);
-        tma_load_2d(sX + j * 16384, &tmap_x, &bar.xfull[j], kx0 + j * 64, m0);
+      for (int j = 0; j < nk; ++j) {
+        const int slot = j % kNXS;
+        if (j >= kNXS) mbar_wait(&bar.xempty[slot], ((j / kNXS) - 1) & 1);
+        mbar_expect_tx(&bar.xfull[slot], p.box_rows * 128);
+        tma_load_2d(sX + slot * 16384, &tmap_x, &bar.xfull[slot], kx0 + j * 64, m0);
       }
+    }
+  } else if (warp == kWarpCp) {
+    // ===================== A producer (copy): smem ring -> TMEM columns [32 j, 32 j + 32)
+    if (lane == 0) {
       for (int j = 0; j < nk; ++j) {
         const int slot = j % kNXS;
         mbar_wait(&bar.xfull[slot], (j / kNXS) & 1);
@@ -201,16 +206,12 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
 #pragma unroll
         for (int s = 0; s < 4; ++s)
           tmem_cp_128x256b(tbase + j * 32 + s * 8, make_sdesc(src + s * 32, 16, 1024, kLayoutSW128));
-        mma_commit(&bar.afill[j]);
-        mma_commit(&bar.xempty[slot]);
-        // refill the slot of the PREVIOUS chunk (its copy has had time to finish) with chunk j-1+NXS
-        const int jr = j - 1;
-        if (jr >= 0 && jr + kNXS < nk) {
-          const int rs = jr % kNXS;
-          mbar_wait(&bar.xempty[rs], (jr / kNXS) & 1);
-          mbar_expect_tx(&bar.xfull[rs], p.box_rows * 128);
-          tma_load_2d(sX + rs * 16384, &tmap_x, &bar.xfull[rs], kx0 + (jr + kNXS) * 64, m0);
-        }
+        mma_commit(&bar.afill[j]);       // chunk j readable by the MMA warps
+        mma_commit(&bar.xempty[slot]);   // smem slot free for the TMA thread
+#ifdef ET_TIMELINE
+        mbar_wait(&bar.afill[j], 0);
+        ET_TL(2 + j);
+#endif
       }
     }
   } else if (warp == kWarpB) {
@@ -226,7 +227,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         const int slot = c % kNBS;
         if (c >= kNBS) {
           const int end_tile = pb + (c - kNBS + 1) * kChunkTiles;
-          while (tl + 1 < nrows && rp[pc.i0 + tl + 1] < end_tile) ++tl;
+          while (tl + 1 < nrows && bar.rptr[tl + 1] + pb < end_tile) ++tl;
           const int full = (tl + 1) / kMmaWarps, rem = (tl + 1) % kMmaWarps;
           const int need0 = 4 * full + min(max(rem, 0), 4);
           const int need1 = 4 * full + min(max(rem - 4, 0), 4);
@@ -234,9 +235,15 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           while (ld_acquire_shared(&bar.rows_seen[1]) < need1) {}
         }
         const int nt = min(kChunkTiles, pe - pb - c * kChunkTiles);
-        mbar_expect_tx(&bar.bfull[c], nt * 512);
+        // tile columns: copy from the 16-byte aligned start at or below the chunk's first entry
+        // (tile_col is allocated with 16 bytes of slack, et_prune_pack_query)
+        const int first = pb + c * kChunkTiles, off = first & 3;
+        const int col_bytes = ((off + nt) * 4 + 15) & ~15;
+        mbar_expect_tx(&bar.bfull[c], nt * 512 + col_bytes);
         bulk_load(sB + slot * (kChunkTiles * 512), vals + (size_t)c * kChunkTiles * 512, nt * 512, &bar.bfull[c]);
+        bulk_load(&bar.tcol[slot][0], sg.tile_col + (first - off), col_bytes, &bar.bfull[c]);
       }
+      ET_TL(14);
     }
   } else if (warp < kMmaWarps) {
     // ===================== MMA warps: warp w issues the chains of tile rows w, w+8, w+16, ...
@@ -253,67 +260,154 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         mbar_wait_warp(&bar.acc_empty[warp], (k - 1) & 1);
         tc_fence_after();
       }
-      const int i = pc.i0 + t;
-      const int p0 = rp[i], p1 = rp[i + 1];
-      for (int base = p0; base < p1; base += 32) {
-        const int mycol = (base + lane < p1) ? sg.tile_col[base + lane] : 0;
-        const int n = min(32, p1 - base);
-        for (int u = 0; u < n; ++u) {
-          const int pp = base + u;
-          const int kc = __shfl_sync(0xffffffffu, mycol, u) - kbase;
-          const int c = (pp - pb) / kChunkTiles;
-          if (c != cur_chunk) {
-            mbar_wait_warp(&bar.bfull[c], 0);
-            cur_chunk = c;
-            tc_fence_after();
-          }
-          const int ach = kc >> 2;
-          if (ach > a_ready) {
-            mbar_wait_warp(&bar.afill[ach], 0);
-            a_ready = ach;
-            tc_fence_after();
-          }
-          const uint32_t baddr = sB_u32 + (c % kNBS) * (kChunkTiles * 512) + ((pp - pb) % kChunkTiles) * 512;
-          mma_ts_warp(d_tmem, tbase + kc * 8, make_sdesc(baddr, 128, 256, kLayoutNone), idesc, pp != p0);
+      if (lane == 0) ET_TL(16 + 8 * warp + 2 * k);
+      const int q0 = bar.rptr[t], q1 = bar.rptr[t + 1];   // this row's tiles, relative to pb
+      for (int q = q0; q < q1; ++q) {
+        const int c = q / kChunkTiles;
+        if (c != cur_chunk) {
+          mbar_wait_warp(&bar.bfull[c], 0);
+          cur_chunk = c;
+          tc_fence_after();
         }
+        const int slot = c % kNBS;
+        const int kc = bar.tcol[slot][((pb + c * kChunkTiles) & 3) + q % kChunkTiles] - kbase;
+        const int ach = kc >> 2;
+        if (ach > a_ready) {
+          mbar_wait_warp(&bar.afill[ach], 0);
+          a_ready = ach;
+          tc_fence_after();
+        }
+        const uint32_t baddr = sB_u32 + slot * (kChunkTiles * 512) + (q % kChunkTiles) * 512;
+        if (warp == 0 && k == 1 && lane == 0 && q - q0 < 24) ET_TL(300 + (q - q0));
+        mma_ts_warp(d_tmem, tbase + kc * 8, make_sdesc(baddr, 128, 256, kLayoutNone), idesc, q != q0);
       }
       mma_commit_warp(&bar.acc_full[warp]);   // fires when this row's MMAs are complete
+      if (lane == 0) ET_TL(16 + 8 * warp + 2 * k + 1);
     }
   } else {
     // ===================== epilogue warps: group g drains the accumulators of MMA warps 4g..4g+3
-    const int e = warp - kMmaWarps;
-    const int g = e >> 2;
+    const int g = (warp - kMmaWarps) >> 2;
     const int quarter = warp & 3;               // TMEM lane quarter this warp may access
-    const int row_g = m0 + quarter * 32 + lane;
-    int seen = 0;
+    // Per round: wait for the group's 4 accumulators (rows 8k + 4g + a), read all 64 columns with
+    // one TMEM load, release them to the MMA warps, THEN do the bias / activation / store math (so
+    // an MMA warp never waits for another row's epilogue arithmetic).
     for (int k = 0; k < nrounds; ++k) {
-#pragma unroll 1
-      for (int a = 0; a < 4; ++a) {
-        const int w = g * 4 + a;
-        const int t = k * kMmaWarps + w;
-        if (t >= nrows) break;
-        mbar_wait_warp(&bar.acc_full[w], k & 1);
-        tc_fence_after();
-        if (quarter == 0 && lane == 0) st_release_shared(&bar.rows_seen[g], ++seen);   // row's B tiles free
-        uint32_t r[16];
-        tmem_ld16(tbase + kAccCol + w * 16 + ((uint32_t)(quarter * 32) << 16), r);
-        tmem_ld_wait();
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&bar.acc_empty[w]);   // accumulator may take its next row
-        const int i = pc.i0 + t;
-        float acc[16];
-        const bool empty_row = rp[i + 1] == rp[i];      // fully pruned tile row: never written
-#pragma unroll
-        for (int c = 0; c < 16; ++c) acc[c] = empty_row ? 0.f : __uint_as_float(r[c]);
-        if (row_g < p.M) epilogue_store<kEpi, kBF16>(p, sg, row_g, i * 16, acc, z);
+      const int t0 = k * kMmaWarps + g * 4;   // first row of this group's quad in round k
+      if (t0 >= nrows) break;
+      const int na = min(4, nrows - t0);
+      for (int a = 0; a < na; ++a) {
+        mbar_wait_warp(&bar.acc_full[g * 4 + a], k & 1);
+        if (k == 1 && g == 0 && a == 0 && quarter == 0 && lane == 0) ET_TL(330);
       }
+      tc_fence_after();
+      if (quarter == 0 && lane == 0)
+        st_release_shared(&bar.rows_seen[g], k * 4 + na);   // rows' MMAs complete: their B tiles are free
+      uint32_t r[64];
+      tmem_ld32(tbase + kAccCol + g * 64 + ((uint32_t)(quarter * 32) << 16), *reinterpret_cast<uint32_t(*)[32]>(r));
+      tmem_ld32(tbase + kAccCol + g * 64 + 32 + ((uint32_t)(quarter * 32) << 16),
+                *reinterpret_cast<uint32_t(*)[32]>(r + 32));
+      tmem_ld_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0)
+        for (int a = 0; a < na; ++a) mbar_arrive(&bar.acc_empty[g * 4 + a]);
+      if (quarter == 0 && lane == 0) ET_TL(96 + 2 * t0);
+      // math: bias / scale / activation on the quad's 64 columns of this thread's token row
+      float v[64];
+#pragma unroll
+      for (int a = 0; a < 4; ++a) {
+        const int t = t0 + min(a, na - 1);
+        const bool empty_row = a >= na || bar.rptr[t + 1] == bar.rptr[t];   // never written: zero
+        float b[16];
+        if constexpr (kEpi != ET_EPI_F32) {
+#pragma unroll
+          for (int c = 0; c < 8; ++c) {
+            const float2 f = unpack2<kBF16>(bar.bias_s[t * 8 + c]);
+            b[2 * c] = f.x;
+            b[2 * c + 1] = f.y;
+          }
+        }
+#pragma unroll
+        for (int c = 0; c < 16; ++c) {
+          float x = empty_row ? 0.f : __uint_as_float(r[a * 16 + c]);
+          if constexpr (kEpi != ET_EPI_F32) {
+            x += b[c];
+            if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
+              if (sg.apply_scale) x *= sg.scale;
+            } else if constexpr (kEpi == ET_EPI_BIAS_GELU) {
+              x = gelu_erf(x);
+            } else if constexpr (kEpi == ET_EPI_BIAS_RELU) {
+              x = fmaxf(x, 0.0f);
+            }
+          }
+          v[a * 16 + c] = x;
+        }
+      }
+      // store: registers -> this warp's 32-row staging tile (128 B rows, SWIZZLE_128B, conflict-free)
+      // -> one TMA tensor store per 128-byte column block (clipped at M by the tensor map)
+      uint8_t* st = sStage + (warp - kMmaWarps) * 4096;
+      const int col0 = sg.out_col + (pc.i0 + t0) * 16;
+      const int row0 = m0 + quarter * 32;
+      constexpr int kPasses = kEpi == ET_EPI_F32 ? 2 : 1;   // fp32: 32 columns (128 B) per pass
+      if (na == 4) {
+#pragma unroll
+        for (int ps = 0; ps < kPasses; ++ps) {
+          if (lane == 0) bulk_wait_group_read<0>();   // previous store finished reading the staging tile
+          __syncwarp();
+#pragma unroll
+          for (int ch = 0; ch < 8; ++ch) {   // 8 x 16-byte chunks of this row's 128 bytes
+            uint4 u;
+            if constexpr (kEpi == ET_EPI_F32) {
+              const float* f = v + ps * 32 + ch * 4;
+              u = make_uint4(__float_as_uint(f[0]), __float_as_uint(f[1]), __float_as_uint(f[2]),
+                             __float_as_uint(f[3]));
+            } else {
+              const float* f = v + ch * 8;
+              u = make_uint4(pack2<kBF16>(f[0], f[1]), pack2<kBF16>(f[2], f[3]), pack2<kBF16>(f[4], f[5]),
+                             pack2<kBF16>(f[6], f[7]));
+            }
+            *reinterpret_cast<uint4*>(st + lane * 128 + ((ch ^ (lane & 7)) << 4)) = u;
+          }
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) {
+            if constexpr (kEpi == ET_EPI_F32) tma_store_3d(&tmap_y, st, col0 + ps * 32, row0, z);
+            else tma_store_2d(&tmap_y, st, col0, row0);
+            bulk_commit_group();
+          }
+        }
+      } else {
+        // partial quad (last rows of a segment): direct stores of the valid 16-column groups only,
+        // so nothing is written into the neighbouring segment's columns
+        const int row = row0 + lane;
+        if (row < p.M) {
+          for (int a = 0; a < na; ++a) {
+            if constexpr (kEpi == ET_EPI_F32) {
+              float* y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row * p.ldy + col0 + a * 16;
+#pragma unroll
+              for (int c = 0; c < 16; c += 4)
+                *reinterpret_cast<float4*>(y + c) = make_float4(v[a * 16 + c], v[a * 16 + c + 1], v[a * 16 + c + 2],
+                                                               v[a * 16 + c + 3]);
+            } else {
+              uint16_t* y = static_cast<uint16_t*>(p.Y) + (size_t)row * p.ldy + col0 + a * 16;
+              const float* f = v + a * 16;
+              *reinterpret_cast<uint4*>(y) = make_uint4(pack2<kBF16>(f[0], f[1]), pack2<kBF16>(f[2], f[3]),
+                                                        pack2<kBF16>(f[4], f[5]), pack2<kBF16>(f[6], f[7]));
+              *reinterpret_cast<uint4*>(y + 8) = make_uint4(pack2<kBF16>(f[8], f[9]), pack2<kBF16>(f[10], f[11]),
+                                                            pack2<kBF16>(f[12], f[13]), pack2<kBF16>(f[14], f[15]));
+            }
+          }
+        }
+      }
+      if (quarter == 0 && lane == 0) ET_TL(96 + 2 * t0 + 1);
     }
   }
 
+  if (warp >= kMmaWarps && warp < kMmaWarps + 8 && lane == 0) bulk_wait_group<0>();   // epilogue stores done
   __syncwarp();   // producer warps: lane 0 ran the loops alone; reconverge before the block barrier
   tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) ET_TL(255);
   if (warp == kWarpB) {
     __syncwarp();
     tc_fence_after();
@@ -340,7 +434,8 @@ EncodeTiledFn get_encode() {
 }
 
 template <int kEpi, bool kBF16>
-et_status launch_typed(const CUtensorMap& tm, const Params& prm, dim3 grid, cudaStream_t stream) {
+et_status launch_typed(const CUtensorMap& tm, const CUtensorMap& tmy, const Params& prm, dim3 grid,
+                       cudaStream_t stream) {
   auto kern = tsgemm_kernel<kEpi, kBF16>;
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
@@ -348,7 +443,7 @@ et_status launch_typed(const CUtensorMap& tm, const Params& prm, dim3 grid, cuda
     attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   });
   ET_CUDA(attr_err);
-  kern<<<grid, kThreads, kSmemBytes, stream>>>(tm, prm);
+  kern<<<grid, kThreads, kSmemBytes, stream>>>(tm, tmy, prm);
   count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
@@ -371,6 +466,21 @@ et_status make_tmap_2d(CUtensorMap* tm, const void* base, et_dtype dtype, uint64
                    swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return ET_OK;
+}
+
+et_status make_tmap_3d_f32(CUtensorMap* tm, void* base, uint64_t cols, uint64_t rows, uint64_t planes,
+                           uint32_t box_cols, uint32_t box_rows) {
+  EncodeTiledFn enc = get_encode();
+  if (!enc) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[3] = {cols, rows, planes};
+  cuuint64_t strides[2] = {cols * 4, cols * rows * 4};
+  cuuint32_t box[3] = {box_cols, box_rows, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = enc(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, base, dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled (3d) failed (%d)", (int)r);
   return ET_OK;
 }
 
@@ -421,17 +531,23 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     for (;;) {
       bool ok = true;
       for (int k = 0; k < ps && ok; ++k) {
-        const int i0 = (int)((long long)gs.tile_rows * k / ps), i1 = (int)((long long)gs.tile_rows * (k + 1) / ps);
-        ok = (long long)(i1 - i0) * (a.K / 16) <= (long long)kMaxBChunks * kChunkTiles;
+        const int q4 = (gs.tile_rows + 3) / 4;
+        const int i0 = std::min(gs.tile_rows, 4 * (int)((long long)q4 * k / ps));
+        const int i1 = std::min(gs.tile_rows, 4 * (int)((long long)q4 * (k + 1) / ps));
+        ok = (long long)(i1 - i0) * (std::min(a.K, 768) / 16) <= (long long)kMaxBChunks * kChunkTiles &&
+             i1 - i0 <= kMaxRows;
       }
-      if (ok || ps >= gs.tile_rows) break;
+      if (ok || ps >= (gs.tile_rows + 3) / 4) break;
       ++ps;
     }
+    ps = std::min(ps, (gs.tile_rows + 3) / 4);   // no empty pieces
     for (int k = 0; k < ps; ++k) {
       if (np >= kMaxPieces) return fail(ET_ERR_INTERNAL, "tile GEMM: too many pieces");
       prm.piece[np].seg = (int16_t)s;
-      prm.piece[np].i0 = (int16_t)((long long)gs.tile_rows * k / ps);
-      prm.piece[np].i1 = (int16_t)((long long)gs.tile_rows * (k + 1) / ps);
+      // piece boundaries on multiples of 4 tile rows (an epilogue quad never straddles two CTAs)
+      const int q4 = (gs.tile_rows + 3) / 4;
+      prm.piece[np].i0 = (int16_t)std::min(gs.tile_rows, 4 * (int)((long long)q4 * k / ps));
+      prm.piece[np].i1 = (int16_t)std::min(gs.tile_rows, 4 * (int)((long long)q4 * (k + 1) / ps));
       ++np;
     }
   }
@@ -439,21 +555,37 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   CUtensorMap tm;   // the K offset k0 is folded into the base address
   ET_TRY(make_tmap_2d(&tm, static_cast<const uint8_t*>(a.X) + (size_t)a.k0 * 2, a.dtype, (uint64_t)a.M,
                       (uint64_t)a.K, (uint64_t)a.ldx, 64, (uint32_t)prm.box_rows, true));
+  // output tensor map: [M, ldy] in the operand dtype, box 64 cols x 32 rows (one epilogue warp's
+  // staging tile); fp32 partials: [kparts, M, ldy], box 32 x 32 x 1.  SWIZZLE_128B staging.
+  CUtensorMap tmy;
+  if (a.epi == ET_EPI_F32) {
+    ET_TRY(make_tmap_3d_f32(&tmy, a.Y, (uint64_t)a.ldy, (uint64_t)a.M, (uint64_t)kparts, 32,
+                            a.M < 32 ? (uint32_t)a.M : 32u));
+  } else {
+    ET_TRY(make_tmap_2d(&tmy, a.Y, a.dtype, (uint64_t)a.M, (uint64_t)a.ldy, (uint64_t)a.ldy, 64,
+                        a.M < 32 ? (uint32_t)a.M : 32u, true));
+  }
   dim3 grid(np, mblocks, kparts);
   const bool bf = a.dtype == ET_BF16;
   switch (a.epi) {
-    case ET_EPI_BIAS: return bf ? launch_typed<ET_EPI_BIAS, true>(tm, prm, grid, stream)
-                                : launch_typed<ET_EPI_BIAS, false>(tm, prm, grid, stream);
-    case ET_EPI_BIAS_SCALE: return bf ? launch_typed<ET_EPI_BIAS_SCALE, true>(tm, prm, grid, stream)
-                                      : launch_typed<ET_EPI_BIAS_SCALE, false>(tm, prm, grid, stream);
-    case ET_EPI_BIAS_GELU: return bf ? launch_typed<ET_EPI_BIAS_GELU, true>(tm, prm, grid, stream)
-                                     : launch_typed<ET_EPI_BIAS_GELU, false>(tm, prm, grid, stream);
-    case ET_EPI_BIAS_RELU: return bf ? launch_typed<ET_EPI_BIAS_RELU, true>(tm, prm, grid, stream)
-                                     : launch_typed<ET_EPI_BIAS_RELU, false>(tm, prm, grid, stream);
-    case ET_EPI_F32: return bf ? launch_typed<ET_EPI_F32, true>(tm, prm, grid, stream)
-                               : launch_typed<ET_EPI_F32, false>(tm, prm, grid, stream);
+    case ET_EPI_BIAS: return bf ? launch_typed<ET_EPI_BIAS, true>(tm, tmy, prm, grid, stream)
+                                : launch_typed<ET_EPI_BIAS, false>(tm, tmy, prm, grid, stream);
+    case ET_EPI_BIAS_SCALE: return bf ? launch_typed<ET_EPI_BIAS_SCALE, true>(tm, tmy, prm, grid, stream)
+                                      : launch_typed<ET_EPI_BIAS_SCALE, false>(tm, tmy, prm, grid, stream);
+    case ET_EPI_BIAS_GELU: return bf ? launch_typed<ET_EPI_BIAS_GELU, true>(tm, tmy, prm, grid, stream)
+                                     : launch_typed<ET_EPI_BIAS_GELU, false>(tm, tmy, prm, grid, stream);
+    case ET_EPI_BIAS_RELU: return bf ? launch_typed<ET_EPI_BIAS_RELU, true>(tm, tmy, prm, grid, stream)
+                                     : launch_typed<ET_EPI_BIAS_RELU, false>(tm, tmy, prm, grid, stream);
+    case ET_EPI_F32: return bf ? launch_typed<ET_EPI_F32, true>(tm, tmy, prm, grid, stream)
+                               : launch_typed<ET_EPI_F32, false>(tm, tmy, prm, grid, stream);
   }
   return fail(ET_ERR_INVALID_ARG, "tile GEMM: bad epilogue %d", (int)a.epi);
 }
+
+#ifdef ET_TIMELINE
+extern "C" int et_diag_gemm_timeline(unsigned long long* host_out) {
+  return cudaMemcpyFromSymbol(host_out, g_timeline, sizeof(g_timeline)) == cudaSuccess ? 0 : 4;
+}
+#endif
 
 }  // namespace et
