@@ -64,7 +64,7 @@ mma_probe_kernel(const __half* __restrict__ A, const __half* __restrict__ B, flo
 
   if (warp == 0) tmem_alloc<512>(&tmem_base_s);
   if (t == 0) {
-    mbar_init(&bar, issue_mode >= 2 ? issue_mode : 1);
+    mbar_init(&bar, issue_mode >= 100 ? issue_mode - 100 : (issue_mode >= 2 ? issue_mode : 1));
     fence_mbar_init();
   }
   tc_fence_before();
@@ -87,6 +87,12 @@ mma_probe_kernel(const __half* __restrict__ A, const __half* __restrict__ B, flo
       if (blockIdx.x == 0) cycles[gridDim.x] = clock64() - c0;
     }
   }
+  if (issue_mode >= 100 && warp < 4) {   // shared-accumulator mode: pre-zero D (this warp's lanes)
+    uint32_t zr[16];
+    for (int i = 0; i < 16; ++i) zr[i] = 0u;
+    for (int c = 0; c < N * n_acc; c += 16) tmem_st16(tbase + ((uint32_t)(warp * 32) << 16) + c, zr);
+    tmem_st_wait();
+  }
   if (a_mode == 1 && warp < 4) {
     // A row t -> TMEM lane t, columns [256, 288): 2 halves per 32-bit column, low half = even k
     uint32_t r[32];
@@ -100,7 +106,8 @@ mma_probe_kernel(const __half* __restrict__ A, const __half* __restrict__ B, flo
   tc_fence_after();
 
   // issue_mode 0: thread 0; 1: warp 0; k >= 2: warps [0, k) each issue accumulators a = w (mod k)
-  const bool issuer = issue_mode == 0 ? (t == 0) : issue_mode == 1 ? (warp == 0) : (warp < issue_mode);
+  const int nissue = issue_mode >= 100 ? issue_mode - 100 : issue_mode;
+  const bool issuer = issue_mode == 0 ? (t == 0) : issue_mode == 1 ? (warp == 0) : (warp < nissue);
   if (issuer) {
     const uint32_t idesc = make_idesc_f16(128, N, 0, 0, b_mode == 2 ? 1 : 0);
     uint64_t adesc[4], bdesc[4];
@@ -113,7 +120,13 @@ mma_probe_kernel(const __half* __restrict__ A, const __half* __restrict__ B, flo
     // issue_mode 2: warp w issues accumulators a = w, w+4, ... (n_acc % 4 == 0)
     const int a0 = issue_mode >= 2 ? warp : 0, astep = issue_mode >= 2 ? issue_mode : 1;
     long long t0 = clock64();
-    if (issue_mode == 0) {
+    if (issue_mode >= 100) {
+      const int a = warp % n_acc;
+      for (int it = 0; it < iters; ++it)
+#pragma unroll
+        for (int s = 0; s < 4; ++s) mma_ts_warp(tbase + a * N, tbase + a_col + s * 8, bdesc[s], idesc, 1u);
+      mma_commit_warp(&bar);
+    } else if (issue_mode == 0) {
       if (a_mode != 0) {
         for (int it = 0; it < iters; ++it)
 #pragma unroll
@@ -174,7 +187,8 @@ extern "C" int et_diag_mma_probe(const void* A, const void* B, float* D, int N, 
   if (n_acc < 1 || N * n_acc > (a_mode != 0 ? 448 : 512)) return 1;
   if (b_mode == 2 && N % 64) return 1;
   if (b_mode == 2 && N > 128) return 1;
-  if (issue_mode >= 2 && (n_acc % issue_mode || issue_mode > 16)) return 1;
+  if (issue_mode >= 2 && issue_mode < 100 && (n_acc % issue_mode || issue_mode > 16)) return 1;
+  if (issue_mode >= 100 && (issue_mode - 100 > 16 || (issue_mode - 100) % n_acc)) return 1;
   const size_t smem = 16384 + 32768 + 1024;
   cudaFuncSetAttribute(et::mma_probe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   et::mma_probe_kernel<<<grid, 512, smem, (cudaStream_t)stream>>>(

@@ -262,24 +262,46 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       }
       if (lane == 0) ET_TL(16 + 8 * warp + 2 * k);
       const int q0 = bar.rptr[t], q1 = bar.rptr[t + 1];   // this row's tiles, relative to pb
-      for (int q = q0; q < q1; ++q) {
-        const int c = q / kChunkTiles;
+      // the row's tiles lie in chunks [q0 / 32, (q1 - 1) / 32]: wait for each once, then read the
+      // tile columns lane-parallel and issue the MMAs from register broadcasts
+      for (int qb = q0; qb < q1;) {
+        const int c = qb / kChunkTiles;
+        const int qe = min(q1, (c + 1) * kChunkTiles);   // tiles of this row inside chunk c
         if (c != cur_chunk) {
           mbar_wait_warp(&bar.bfull[c], 0);
           cur_chunk = c;
           tc_fence_after();
         }
         const int slot = c % kNBS;
-        const int kc = bar.tcol[slot][((pb + c * kChunkTiles) & 3) + q % kChunkTiles] - kbase;
-        const int ach = kc >> 2;
-        if (ach > a_ready) {
-          mbar_wait_warp(&bar.afill[ach], 0);
-          a_ready = ach;
+        const int coff = (pb + c * kChunkTiles) & 3;
+        const int n = qe - qb;
+        const int mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
+        int maxcol = mycol;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) maxcol = max(maxcol, __shfl_xor_sync(0xffffffffu, maxcol, o));
+        if ((maxcol >> 2) > a_ready) {   // all A chunks this segment needs (afill[j] implies all < j)
+          mbar_wait_warp(&bar.afill[maxcol >> 2], 0);
+          a_ready = maxcol >> 2;
           tc_fence_after();
         }
-        const uint32_t baddr = sB_u32 + slot * (kChunkTiles * 512) + (q % kChunkTiles) * 512;
-        if (warp == 0 && k == 1 && lane == 0 && q - q0 < 24) ET_TL(300 + (q - q0));
-        mma_ts_warp(d_tmem, tbase + kc * 8, make_sdesc(baddr, 128, 256, kLayoutNone), idesc, q != q0);
+        // B descriptor of tile u: start address field advances by 512 B / 16 = 32 per tile
+        const uint64_t bd0 = make_sdesc(sB_u32 + slot * (kChunkTiles * 512) + (qb % kChunkTiles) * 512, 128, 256,
+                                        kLayoutNone);
+        const uint32_t blo = (uint32_t)bd0, bhi = (uint32_t)(bd0 >> 32);
+        const uint32_t acol = tbase + (uint32_t)(mycol * 8);   // this lane's tile: its A columns
+        int u = 0;
+        for (; u + 4 <= n; u += 4) {
+          if (warp == 0 && k == 1 && lane == 0 && qb + u - q0 < 24) ET_TL(300 + (qb + u - q0));
+          mma_ts_warp_x4(d_tmem, __shfl_sync(0xffffffffu, acol, u), __shfl_sync(0xffffffffu, acol, u + 1),
+                         __shfl_sync(0xffffffffu, acol, u + 2), __shfl_sync(0xffffffffu, acol, u + 3),
+                         blo + 32 * u, blo + 32 * (u + 1), blo + 32 * (u + 2), blo + 32 * (u + 3), bhi, idesc,
+                         (qb + u) != q0);
+        }
+        for (; u < n; ++u) {
+          const uint32_t a = __shfl_sync(0xffffffffu, acol, u);
+          mma_ts_warp_nc(d_tmem, a, ((uint64_t)bhi << 32) | (blo + 32 * u), idesc, (qb + u) != q0);
+        }
+        qb = qe;
       }
       mma_commit_warp(&bar.acc_full[warp]);   // fires when this row's MMAs are complete
       if (lane == 0) ET_TL(16 + 8 * warp + 2 * k + 1);

@@ -198,9 +198,34 @@ __device__ __forceinline__ void mma_ts_warp(uint32_t d_tmem, uint32_t a_tmem, ui
   asm volatile(
       "{\n .reg .pred p, e;\n .reg .b32 rx;\n elect.sync rx|e, 0xffffffff;\n setp.ne.b32 p, %4, 0;\n"
       " @e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(d_tmem),
-      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
-      : "memory");
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate));
 }
+// Same without a compiler memory clobber: ordered only against other volatile asm (barrier waits,
+// commits), so the compiler may schedule the next iteration's ordinary loads around it.
+__device__ __forceinline__ void mma_ts_warp_nc(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                               uint32_t accumulate) {
+  asm volatile(
+      "{\n .reg .pred p, e;\n .reg .b32 rx;\n elect.sync rx|e, 0xffffffff;\n setp.ne.b32 p, %4, 0;\n"
+      " @e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate));
+}
+// Four TS MMAs into one accumulator under a single elect (cuts per-MMA issue overhead).  The B
+// descriptors differ only in the start-address field: b_lo[i] are the low 32 bits, b_hi shared.
+// acc0: accumulate flag of the FIRST of the four (the other three always accumulate).
+__device__ __forceinline__ void mma_ts_warp_x4(uint32_t d_tmem, uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
+                                               uint32_t b0, uint32_t b1, uint32_t b2, uint32_t b3, uint32_t b_hi,
+                                               uint32_t idesc, uint32_t acc0) {
+  asm volatile(
+      "{\n .reg .pred p, e;\n .reg .b32 rx;\n .reg .b64 d0, d1, d2, d3;\n"
+      " elect.sync rx|e, 0xffffffff;\n setp.ne.b32 p, %11, 0;\n"
+      " mov.b64 d0, {%5, %9};\n mov.b64 d1, {%6, %9};\n mov.b64 d2, {%7, %9};\n mov.b64 d3, {%8, %9};\n"
+      " @e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d0, %10, p;\n"
+      " @e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], d1, %10, 1;\n"
+      " @e tcgen05.mma.cta_group::1.kind::f16 [%0], [%3], d2, %10, 1;\n"
+      " @e tcgen05.mma.cta_group::1.kind::f16 [%0], [%4], d3, %10, 1;\n}\n" ::"r"(d_tmem),
+      "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1), "r"(b2), "r"(b3), "r"(b_hi), "r"(idesc), "r"(acc0));
+}
+
 __device__ __forceinline__ void mma_commit_warp(uint64_t* bar) {
   asm volatile(
       "{\n .reg .pred e;\n .reg .b32 rx;\n elect.sync rx|e, 0xffffffff;\n"
