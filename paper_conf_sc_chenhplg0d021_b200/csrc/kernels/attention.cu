@@ -29,12 +29,32 @@
 
 namespace et {
 
+#ifdef ET_TIMELINE
+__device__ unsigned long long g_attn_tl[64];
+__device__ __forceinline__ unsigned long long gtime_a() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define ET_TLA(slot)                                                                                  \
+  do {                                                                                                \
+    if (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0) g_attn_tl[(slot)] = gtime_a();          \
+  } while (0)
+extern "C" int et_diag_attn_timeline(unsigned long long* host_out) {
+  return cudaMemcpyFromSymbol(host_out, g_attn_tl, sizeof(g_attn_tl)) == cudaSuccess ? 0 : 4;
+}
+#else
+#define ET_TLA(slot) do {} while (0)
+#endif
+
 et_status make_tmap_2d(CUtensorMap* tm, const void* base, et_dtype dtype, uint64_t rows, uint64_t cols,
                        uint64_t ld_elems, uint32_t box_cols, uint32_t box_rows, bool swizzle128);
+et_status make_tmap_2d_sw64(CUtensorMap* tm, const void* base, et_dtype dtype, uint64_t rows, uint64_t cols,
+                            uint64_t ld_elems, uint32_t box_cols, uint32_t box_rows);
 
 namespace {
 
-constexpr int kThreads = 192;
+constexpr int kThreads = 320;   // warp 0 TMA, warp 1 MMA + TMEM, warps 2-9 softmax / epilogue
 constexpr float kLog2e = 1.4426950408889634f;
 
 struct AParams {
@@ -50,12 +70,15 @@ struct AParams {
   int dv_max;               // MMA N for P.V (multiple of 16, <= kDK)
   float scale_log2;         // scale * log2(e)
   int box_rows;             // TMA box height: min(128, total rows)
+  int tma_store;            // Z written through TMA stores (dense V layout, seq_len % 32 == 0)
 };
 
 template <int kDK>
 struct Cfg {
   static constexpr int kTiles = kDK / 64;            // 64-wide SW128 tiles per 128-row operand
   static constexpr int kOpBytes = 128 * kDK * 2;     // one 128-row Q / K / V block
+  static constexpr int kHalf = kDK / 2;              // O columns per softmax thread
+  static constexpr int kStageBytes = 32 * kHalf * 2; // per softmax warp: 32 rows x kHalf fp16
 };
 
 __device__ __forceinline__ float ex2(float x) {
@@ -64,18 +87,28 @@ __device__ __forceinline__ float ex2(float x) {
   return y;
 }
 
-template <bool kBF16, int kDK, bool kLong>
+template <int kCols>
+__device__ __forceinline__ void tmem_alloc_n(uint32_t* slot) { tmem_alloc<kCols>(slot); }
+
+// kNKB: score blocks resident in TMEM (short form: 1 => seq_len <= 128, 2 => <= 256; long form: the
+// two S buffers).  TMEM: S [0, 128 kNKB), P [128 kNKB, 192 kNKB), O [192 kNKB, 192 kNKB + kDK).
+template <bool kBF16, int kDK, bool kLong, int kNKB>
 __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                           const __grid_constant__ CUtensorMap tmap_z,
                                                            const __grid_constant__ AParams p) {
   using C = Cfg<kDK>;
-  constexpr int kStages = 2;   // K/V ring (the short form holds its <= 2 blocks resident)
+  constexpr int kS = 0, kP = 128 * kNKB, kO = 192 * kNKB;
+  constexpr uint32_t kCols = (kO + kDK) <= 256 ? 256u : 512u;
   if (p.v_width && p.v_width[p.head_begin + blockIdx.y] == 0) return;   // every V feature of the head pruned
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
-  uint8_t* sK = sQ + C::kOpBytes;                       // kStages x K block
-  uint8_t* sV = sK + kStages * C::kOpBytes;             // kStages x V block
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sV + kStages * C::kOpBytes);
+  uint8_t* sK = sQ + C::kOpBytes;                // 2 x K block
+  uint8_t* sV = sK + 2 * C::kOpBytes;            // 2 x V block
+  uint8_t* sStage = sV + 2 * C::kOpBytes;        // 8 x epilogue staging
+  float* xmax = reinterpret_cast<float*>(sStage + 8 * C::kStageBytes);   // [2][128] row-max halves
+  float* xsum = xmax + 256;                                               // [2][128] row-sum halves
+  uint64_t* bars = reinterpret_cast<uint64_t*>(xsum + 256);
   uint64_t* q_full = bars + 0;
   uint64_t* kv_full = bars + 1;       // [2]
   uint64_t* kv_empty = bars + 3;      // [2]
@@ -93,20 +126,15 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
   const int b = blockIdx.z;
   const int S = p.S;
   const int len = p.lengths ? p.lengths[b] : S;
-  // keys needed by this query block: [0, kmax)
-  int kmax = len;
+  int kmax = len;                                  // keys needed by this query block: [0, kmax)
   if (p.causal) kmax = min(kmax, qb * 128 + 128);
   const int nkb = (kmax + 127) / 128;
-  const int row0 = b * S;   // first token row of this sequence
+  const int row0 = b * S;                          // first token row of this sequence
   const int qcol = p.q_off + h * kDK, kcol = p.k_off + h * kDK;
-  const int vcol = p.v_off + (p.v_col ? p.v_col[h] : h * kDK);
+  const int vloc = p.v_col ? p.v_col[h] : h * kDK; // packed V column of this head
+  const int vcol = p.v_off + vloc;
   const int vw = p.v_width ? p.v_width[h] : kDK;
-  const int dvn = p.dv_max;   // P.V MMA N
-
-  // TMEM columns
-  constexpr int kS = 0;                    // S: [0, 256) (short: all blocks; long: 2 buffers)
-  constexpr int kP = 256;                  // P: [256, 384) fp16 pairs, 64 columns per 128 keys
-  constexpr int kO = 384;                  // O: [384, 384 + dv)
+  const int dvn = p.dv_max;                        // P.V MMA N
 
   if (p.box_rows < 128) {
     // tiny problem: the TMA box covers fewer than 128 rows; zero the V staging so that the rows
@@ -121,18 +149,20 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
       mbar_init(&kv_full[i], 1);
       mbar_init(&kv_empty[i], 1);
       mbar_init(&s_full[i], 1);
-      mbar_init(&s_free[i], 4);
-      mbar_init(&p_full[i], 4);
+      mbar_init(&s_free[i], 8);
+      mbar_init(&p_full[i], 8);
     }
     mbar_init(o_full, 1);
-    mbar_init(o_free, 4);
+    mbar_init(o_free, 8);
     fence_mbar_init();
   }
-  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  if (threadIdx.x == 0) ET_TLA(0);
+  if (warp == 1) tmem_alloc<kCols>(tmem_slot);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
+  if (threadIdx.x == 0) ET_TLA(1);
 
   if (warp == 0) {
     // ================= TMA producer: Q once, then K/V blocks through a 2-stage ring
@@ -175,16 +205,19 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
     };
     mbar_wait_warp(q_full, 0);
     tc_fence_after();
+    if (lane == 0) ET_TLA(2);
     if constexpr (!kLong) {
-      // short form: all score blocks, then one P.V chain over all keys
+      // short form: every score block, then one P.V chain over all keys
       for (int j = 0; j < nkb; ++j) {
         mbar_wait_warp(&kv_full[j], 0);
         tc_fence_after();
         issue_qk(j, kS + j * 128);
       }
       mma_commit_warp(&s_full[0]);
+      if (lane == 0) ET_TLA(3);
       mbar_wait_warp(&p_full[0], 0);
       tc_fence_after();
+      if (lane == 0) ET_TLA(4);
       for (int j = 0; j < nkb; ++j) issue_pv(j, kP + j * 64, j > 0);
       mma_commit_warp(o_full);
     } else {
@@ -213,80 +246,91 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
       }
     }
   } else {
-    // ================= softmax / epilogue: one thread per query row
-    const int quarter = warp & 3;
-    const int r = quarter * 32 + lane;          // row within the block = TMEM lane
-    const int qi = qb * 128 + r;                // query index within the sequence
+    // ================= softmax / epilogue: two threads per query row, each owning 64 of every
+    // 128 keys (and half of the O columns); row max / sum halves meet in shared memory
+    const int sw = warp - 2;                     // 0..7
+    const int half = sw >> 2;                    // key / O-column half
+    const int quarter = warp & 3;                // TMEM lane quarter this warp may access
+    const int r = quarter * 32 + lane;           // query row within the block = TMEM lane
+    const int qi = qb * 128 + r;                 // query index within the sequence
     const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
-    int kend = len;                             // valid keys: [0, kend)
+    int kend = len;                              // valid keys: [0, kend)
     if (p.causal) kend = min(kend, qi + 1);
     const float sl2 = p.scale_log2;
-    float o[kLong ? kDK : 1];
+    float o[kLong ? C::kHalf : 1];
 #pragma unroll
-    for (int c = 0; c < (kLong ? kDK : 1); ++c) o[c] = 0.f;
-    float l = 0.f;
+    for (int c = 0; c < (kLong ? C::kHalf : 1); ++c) o[c] = 0.f;
+    float lpart = 0.f;                           // this half's share of the row sum
 
     if constexpr (!kLong) {
       mbar_wait_warp(&s_full[0], 0);
       tc_fence_after();
-      // pass 1: row max over valid keys
+      if (threadIdx.x == 64) ET_TLA(5);
       float m = -INFINITY;
       for (int j = 0; j < nkb; ++j) {
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
+        for (int c = 0; c < 2; ++c) {
           uint32_t v[32];
-          tmem_ld32(tbase + lane_off + kS + j * 128 + c * 32, v);
+          const int k0 = j * 128 + half * 64 + c * 32;
+          tmem_ld32(tbase + lane_off + kS + k0, v);
           tmem_ld_wait();
 #pragma unroll
-          for (int t = 0; t < 32; ++t) {
-            const int key = j * 128 + c * 32 + t;
-            if (key < kend) m = fmaxf(m, __uint_as_float(v[t]));
-          }
+          for (int t = 0; t < 32; ++t)
+            if (k0 + t < kend) m = fmaxf(m, __uint_as_float(v[t]));
         }
       }
-      // pass 2: p = exp(s - m) (0 for masked keys), row sum, P -> TMEM (16-bit pairs)
+      xmax[half * 128 + r] = m;
+      named_bar_sync(1, 256);
+      m = fmaxf(m, xmax[(half ^ 1) * 128 + r]);
       const float mb = m * sl2;
       for (int j = 0; j < nkb; ++j) {
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
+        for (int c = 0; c < 2; ++c) {
           uint32_t v[32];
-          tmem_ld32(tbase + lane_off + kS + j * 128 + c * 32, v);
+          const int k0 = j * 128 + half * 64 + c * 32;
+          tmem_ld32(tbase + lane_off + kS + k0, v);
           tmem_ld_wait();
           uint32_t pk[16];
 #pragma unroll
           for (int t = 0; t < 32; t += 2) {
-            const int key = j * 128 + c * 32 + t;
-            const float p0 = key < kend ? ex2(__uint_as_float(v[t]) * sl2 - mb) : 0.f;
-            const float p1 = key + 1 < kend ? ex2(__uint_as_float(v[t + 1]) * sl2 - mb) : 0.f;
-            l += p0 + p1;
+            const float p0 = k0 + t < kend ? ex2(__uint_as_float(v[t]) * sl2 - mb) : 0.f;
+            const float p1 = k0 + t + 1 < kend ? ex2(__uint_as_float(v[t + 1]) * sl2 - mb) : 0.f;
+            lpart += p0 + p1;
             pk[t >> 1] = pack2<kBF16>(p0, p1);
           }
-          tmem_st16(tbase + lane_off + kP + j * 64 + c * 16, pk);
+          tmem_st16(tbase + lane_off + kP + j * 64 + half * 32 + c * 16, pk);
         }
       }
       tmem_st_wait();
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&p_full[0]);
+      if (threadIdx.x == 64) ET_TLA(6);
       mbar_wait_warp(o_full, 0);
       tc_fence_after();
+      if (threadIdx.x == 64) ET_TLA(7);
     } else {
       float m = -INFINITY;
       for (int j = 0; j < nkb; ++j) {
         const int bj = j & 1;
         mbar_wait_warp(&s_full[bj], (j >> 1) & 1);
         tc_fence_after();
-        // pass A: block max over valid keys (S read from TMEM, not kept in registers)
+        // pass A: block max over this half's valid keys, combined with the other half
         float mblk = -INFINITY;
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
+        for (int c = 0; c < 2; ++c) {
           uint32_t v[32];
-          tmem_ld32(tbase + lane_off + kS + bj * 128 + c * 32, v);
+          const int kl = half * 64 + c * 32;
+          tmem_ld32(tbase + lane_off + kS + bj * 128 + kl, v);
           tmem_ld_wait();
 #pragma unroll
           for (int t = 0; t < 32; ++t)
-            if (j * 128 + c * 32 + t < kend) mblk = fmaxf(mblk, __uint_as_float(v[t]));
+            if (j * 128 + kl + t < kend) mblk = fmaxf(mblk, __uint_as_float(v[t]));
         }
+        xmax[half * 128 + r] = mblk;
+        named_bar_sync(1, 256);
+        mblk = fmaxf(mblk, xmax[(half ^ 1) * 128 + r]);
+        named_bar_sync(2, 256);   // both halves read xmax before it is rewritten for the next block
         const float m_new = fmaxf(m, mblk);
         const float alpha = (m == -INFINITY) ? 0.f : ex2((m - m_new) * sl2);
         const float mb = m_new * sl2;
@@ -294,20 +338,21 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
         // pass B: p = exp(s - m_new) -> P(j) in TMEM buffer j&1 (its previous reader PV(j-2)
         // completed before o_full(j-1) was observed)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
+        for (int c = 0; c < 2; ++c) {
           uint32_t v[32];
-          tmem_ld32(tbase + lane_off + kS + bj * 128 + c * 32, v);
+          const int kl = half * 64 + c * 32;
+          tmem_ld32(tbase + lane_off + kS + bj * 128 + kl, v);
           tmem_ld_wait();
           uint32_t pk[16];
 #pragma unroll
           for (int t = 0; t < 32; t += 2) {
-            const int key = j * 128 + c * 32 + t;
+            const int key = j * 128 + kl + t;
             const float p0 = key < kend ? ex2(__uint_as_float(v[t]) * sl2 - mb) : 0.f;
             const float p1 = key + 1 < kend ? ex2(__uint_as_float(v[t + 1]) * sl2 - mb) : 0.f;
             lsum += p0 + p1;
             pk[t >> 1] = pack2<kBF16>(p0, p1);
           }
-          tmem_st16(tbase + lane_off + kP + bj * 64 + c * 16, pk);
+          tmem_st16(tbase + lane_off + kP + bj * 64 + half * 32 + c * 16, pk);
         }
         tmem_st_wait();
         tc_fence_before();
@@ -316,16 +361,16 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
           mbar_arrive(&s_free[bj]);   // S(j) consumed: its buffer may take QK(j+2)
           mbar_arrive(&p_full[bj]);
         }
-        l = l * alpha + lsum;
+        lpart = lpart * alpha + lsum;
         m = m_new;
-        // O += P(j) V(j), rescaled
+        // O += P(j) V(j), rescaled (this thread's half of the O columns)
         mbar_wait_warp(o_full, j & 1);
         tc_fence_after();
 #pragma unroll
-        for (int c = 0; c < kDK; c += 32) {
-          if (c < dvn) {
+        for (int c = 0; c < C::kHalf; c += 32) {
+          if (half * C::kHalf + c < dvn) {
             uint32_t v[32];
-            tmem_ld32(tbase + lane_off + kO + c, v);
+            tmem_ld32(tbase + lane_off + kO + half * C::kHalf + c, v);
             tmem_ld_wait();
 #pragma unroll
             for (int t = 0; t < 32; ++t) o[c + t] = o[c + t] * alpha + __uint_as_float(v[t]);
@@ -337,86 +382,101 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
       }
     }
 
-    // ---- epilogue: Z = O / l in 32-column chunks.  The TMEM loads are warp-collective
-    // (.sync.aligned) and stay outside the per-row condition; only the stores are predicated on
-    // the row lying inside the sequence.
-    {
-      using T = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
-      const bool store = qi < S;
-      const float inv = 1.0f / l;
-      T* zrow = static_cast<T*>(p.Z) + (size_t)(row0 + qi) * p.ld_z;
-      const int vloc = p.v_col ? p.v_col[h] : h * kDK;        // packed V column of this head
-      const int32_t* zm = p.z_map ? p.z_map + vloc : nullptr;  // scatter map (row-pruned W_V)
-      T* z = zrow + h * kDK;
+    // ---- epilogue: Z = O / l.  l = both halves' sums (exchanged through shared memory).  The TMEM
+    // loads are warp-collective and stay outside any per-row condition.
+    xsum[half * 128 + r] = lpart;
+    named_bar_sync(1, 256);
+    const float inv = 1.0f / (lpart + xsum[(half ^ 1) * 128 + r]);
+    using T = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
+    const bool store = qi < S;
+    // TMA path: this warp's 32 rows all lie inside the sequence (S % 32 == 0, so a warp's rows are
+    // either all valid or all beyond the sequence — those must not be written at all)
+    const bool tma_warp = p.tma_store && (qb * 128 + quarter * 32 < S);
+    const int ccol0 = half * C::kHalf;           // first O column of this thread
+    uint8_t* st = sStage + sw * C::kStageBytes;  // 32 rows x kHalf fp16, 64-byte rows (SWIZZLE_64B)
+    T* zrow = static_cast<T*>(p.Z) + (size_t)(row0 + qi) * p.ld_z;
 #pragma unroll
-      for (int c0 = 0; c0 < kDK; c0 += 32) {
-        if (c0 < vw) {
-          float x[32];
-          if constexpr (kLong) {
+    for (int c0 = 0; c0 < C::kHalf; c0 += 32) {
+      if (ccol0 + c0 < vw) {
+        float x[32];
+        if constexpr (kLong) {
 #pragma unroll
-            for (int t = 0; t < 32; ++t) x[t] = o[c0 + t];
-          } else {
-            uint32_t v[32];
-            tmem_ld32(tbase + lane_off + kO + c0, v);
-            tmem_ld_wait();
+          for (int t = 0; t < 32; ++t) x[t] = o[c0 + t];
+        } else {
+          uint32_t v[32];
+          tmem_ld32(tbase + lane_off + kO + ccol0 + c0, v);
+          tmem_ld_wait();
 #pragma unroll
-            for (int t = 0; t < 32; ++t) x[t] = __uint_as_float(v[t]);
+          for (int t = 0; t < 32; ++t) x[t] = __uint_as_float(v[t]);
+        }
+        if (tma_warp) {
+          // 32 columns = 64 bytes per row: 4 x 16-byte chunks, SWIZZLE_64B position c ^ ((row >> 1) & 3)
+#pragma unroll
+          for (int ch = 0; ch < 4; ++ch) {
+            const uint4 u = make_uint4(pack2<kBF16>(x[8 * ch] * inv, x[8 * ch + 1] * inv),
+                                       pack2<kBF16>(x[8 * ch + 2] * inv, x[8 * ch + 3] * inv),
+                                       pack2<kBF16>(x[8 * ch + 4] * inv, x[8 * ch + 5] * inv),
+                                       pack2<kBF16>(x[8 * ch + 6] * inv, x[8 * ch + 7] * inv));
+            *reinterpret_cast<uint4*>(st + (c0 / 32) * 2048 + lane * 64 + ((ch ^ ((lane >> 1) & 3)) << 4)) = u;
           }
-          if (!store) {
-          } else if (zm) {
+        } else if (store && !p.tma_store) {
+          if (p.z_map) {
+            const int32_t* zm = p.z_map + vloc + ccol0 + c0;
 #pragma unroll
             for (int t = 0; t < 32; ++t)
-              if (c0 + t < vw) {
-                const int dst = zm[c0 + t];
+              if (ccol0 + c0 + t < vw) {
+                const int dst = zm[t];
                 if (dst >= 0) {
                   if constexpr (kBF16) zrow[dst] = __float2bfloat16_rn(x[t] * inv);
                   else zrow[dst] = __float2half_rn(x[t] * inv);
                 }
               }
-          } else if ((vw & 7) == 0) {
-#pragma unroll
-            for (int t = 0; t < 32; t += 8) {
-              if (c0 + t < vw) {
-                uint4 u;
-                u.x = pack2<kBF16>(x[t] * inv, x[t + 1] * inv);
-                u.y = pack2<kBF16>(x[t + 2] * inv, x[t + 3] * inv);
-                u.z = pack2<kBF16>(x[t + 4] * inv, x[t + 5] * inv);
-                u.w = pack2<kBF16>(x[t + 6] * inv, x[t + 7] * inv);
-                *reinterpret_cast<uint4*>(z + c0 + t) = u;
-              }
-            }
           } else {
+            T* z = zrow + h * kDK + ccol0 + c0;
 #pragma unroll
-            for (int t = 0; t < 32; ++t)
-              if (c0 + t < vw) {
-                if constexpr (kBF16) z[c0 + t] = __float2bfloat16_rn(x[t] * inv);
-                else z[c0 + t] = __float2half_rn(x[t] * inv);
-              }
+            for (int t = 0; t < 32; t += 8)
+              if (ccol0 + c0 + t < vw)
+                *reinterpret_cast<uint4*>(z + t) = make_uint4(
+                    pack2<kBF16>(x[t] * inv, x[t + 1] * inv), pack2<kBF16>(x[t + 2] * inv, x[t + 3] * inv),
+                    pack2<kBF16>(x[t + 4] * inv, x[t + 5] * inv), pack2<kBF16>(x[t + 6] * inv, x[t + 7] * inv));
           }
         }
       }
     }
+    if (tma_warp) {
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) {
+#pragma unroll
+        for (int c0 = 0; c0 < C::kHalf; c0 += 32)
+          tma_store_2d(&tmap_z, st + (c0 / 32) * 2048, h * kDK + ccol0 + c0, row0 + qb * 128 + quarter * 32);
+        bulk_commit_group();
+        bulk_wait_group<0>();
+      }
+    }
+    if (threadIdx.x == 64) ET_TLA(8);
   }
 
   __syncwarp();
   tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) ET_TLA(9);
   if (warp == 1) {
     __syncwarp();
     tc_fence_after();
-    tmem_dealloc<512>(tbase);
+    tmem_dealloc<kCols>(tbase);
   }
 }
 
-template <bool kBF16, int kDK, bool kLong>
-et_status launch(const CUtensorMap& tm, const AParams& prm, dim3 grid, cudaStream_t stream) {
-  auto kern = attn_kernel<kBF16, kDK, kLong>;
-  const size_t smem = 1024 + (size_t)(1 + 2 * 2) * Cfg<kDK>::kOpBytes + 256;
+template <bool kBF16, int kDK, bool kLong, int kNKB>
+et_status launch(const CUtensorMap& tm, const CUtensorMap& tz, const AParams& prm, dim3 grid, cudaStream_t stream) {
+  auto kern = attn_kernel<kBF16, kDK, kLong, kNKB>;
+  const size_t smem = 1024 + (size_t)5 * Cfg<kDK>::kOpBytes + 8 * Cfg<kDK>::kStageBytes + 2048 + 256;
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [&] { attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); });
   ET_CUDA(attr_err);
-  kern<<<grid, kThreads, smem, stream>>>(tm, prm);
+  kern<<<grid, kThreads, smem, stream>>>(tm, tz, prm);
   count_launch();
   ET_CUDA(cudaGetLastError());
   return ET_OK;
@@ -434,10 +494,10 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   if (!a.long_form && a.seq_len > 256) return fail(ET_ERR_UNSUPPORTED, "attention: short form needs seq_len <= 256");
   if (a.batch <= 0 || a.seq_len <= 0 || a.head_end <= a.head_begin) return ET_OK;
   if (!aligned16(a.qkv) || (a.ld_qkv * 2) % 16) return fail(ET_ERR_INVALID_ARG, "attention: QKV not 16B aligned");
-  CUtensorMap tm;
-  const uint32_t box_rows = (uint64_t)a.batch * a.seq_len < 128 ? (uint32_t)(a.batch * a.seq_len) : 128u;
-  ET_TRY(make_tmap_2d(&tm, a.qkv, a.dtype, (uint64_t)a.batch * a.seq_len, (uint64_t)a.ld_qkv, (uint64_t)a.ld_qkv, 64,
-                      box_rows, true));
+  const uint64_t rows = (uint64_t)a.batch * a.seq_len;
+  const uint32_t box_rows = rows < 128 ? (uint32_t)rows : 128u;
+  CUtensorMap tm, tz;
+  ET_TRY(make_tmap_2d(&tm, a.qkv, a.dtype, rows, (uint64_t)a.ld_qkv, (uint64_t)a.ld_qkv, 64, box_rows, true));
   AParams prm{};
   prm.S = a.seq_len;
   prm.H = a.heads;
@@ -454,16 +514,27 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   prm.causal = a.causal;
   prm.dv_max = a.v_width_max;
   prm.scale_log2 = a.scale * kLog2e;
-  const long long rows = (long long)a.batch * a.seq_len;
-  prm.box_rows = rows < 128 ? (int)rows : 128;
+  prm.box_rows = (int)box_rows;
+  // TMA stores of Z: dense per-head V, every 32-row group inside one sequence, Z 16-byte aligned
+  prm.tma_store = (a.z_map == nullptr && a.v_width == nullptr && a.seq_len % 32 == 0 && rows >= 32 &&
+                   aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
+  if (prm.tma_store) {
+    ET_TRY(make_tmap_2d_sw64(&tz, a.Z, a.dtype, rows, (uint64_t)a.ld_z, (uint64_t)a.ld_z, 32, 32));
+  } else {
+    tz = tm;   // unused
+  }
   dim3 grid((a.seq_len + 127) / 128, a.head_end - a.head_begin, a.batch);
   const bool bf = a.dtype == ET_BF16;
+  const bool lf = a.long_form;
+  const int nkb1 = a.seq_len <= 128;
   if (a.d_k == 64) {
-    if (a.long_form) return bf ? launch<true, 64, true>(tm, prm, grid, stream) : launch<false, 64, true>(tm, prm, grid, stream);
-    return bf ? launch<true, 64, false>(tm, prm, grid, stream) : launch<false, 64, false>(tm, prm, grid, stream);
+    if (lf) return bf ? launch<true, 64, true, 2>(tm, tz, prm, grid, stream) : launch<false, 64, true, 2>(tm, tz, prm, grid, stream);
+    if (nkb1) return bf ? launch<true, 64, false, 1>(tm, tz, prm, grid, stream) : launch<false, 64, false, 1>(tm, tz, prm, grid, stream);
+    return bf ? launch<true, 64, false, 2>(tm, tz, prm, grid, stream) : launch<false, 64, false, 2>(tm, tz, prm, grid, stream);
   }
-  if (a.long_form) return bf ? launch<true, 128, true>(tm, prm, grid, stream) : launch<false, 128, true>(tm, prm, grid, stream);
-  return bf ? launch<true, 128, false>(tm, prm, grid, stream) : launch<false, 128, false>(tm, prm, grid, stream);
+  if (lf) return bf ? launch<true, 128, true, 2>(tm, tz, prm, grid, stream) : launch<false, 128, true, 2>(tm, tz, prm, grid, stream);
+  if (nkb1) return bf ? launch<true, 128, false, 1>(tm, tz, prm, grid, stream) : launch<false, 128, false, 1>(tm, tz, prm, grid, stream);
+  return bf ? launch<true, 128, false, 2>(tm, tz, prm, grid, stream) : launch<false, 128, false, 2>(tm, tz, prm, grid, stream);
 }
 
 }  // namespace et

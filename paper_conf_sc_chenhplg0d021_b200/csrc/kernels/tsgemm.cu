@@ -491,6 +491,21 @@ et_status make_tmap_2d(CUtensorMap* tm, const void* base, et_dtype dtype, uint64
   return ET_OK;
 }
 
+et_status make_tmap_2d_sw64(CUtensorMap* tm, const void* base, et_dtype dtype, uint64_t rows, uint64_t cols,
+                            uint64_t ld_elems, uint32_t box_cols, uint32_t box_rows) {
+  EncodeTiledFn enc = get_encode();
+  if (!enc) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {ld_elems * dtype_size(dtype)};
+  cuuint32_t box[2] = {box_cols, box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUtensorMapDataType dt = dtype == ET_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  CUresult r = enc(tm, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled (sw64) failed (%d)", (int)r);
+  return ET_OK;
+}
+
 et_status make_tmap_3d_f32(CUtensorMap* tm, void* base, uint64_t cols, uint64_t rows, uint64_t planes,
                            uint32_t box_cols, uint32_t box_rows) {
   EncodeTiledFn enc = get_encode();
