@@ -237,13 +237,15 @@ def our_arm(args):
     import paper_conf_sc_chenhplg0d021_b200 as et
     from et_synth import CONFIGS, make_layer, make_lengths, make_x
 
+    from paper_conf_sc_chenhplg0d021_b200.dist import shard_range
     base = CONFIGS[args.config]
     cfg = base                                   # per-rank shard: the config's batch (weak scaling)
     gcfg = base.with_(batch=base.batch * world)  # the global batch, generated identically everywhere
     dtype = cfg.dtype if cfg.dtype != "fp32" else "fp16"
     raws = [make_layer(cfg, l) for l in range(cfg.layers)]
     Xg = make_x(gcfg)
-    X = Xg[rank * cfg.batch:(rank + 1) * cfg.batch]
+    b0, b1 = shard_range(gcfg.batch, world, rank)
+    X = Xg[b0:b1]
     lens = make_lengths(cfg, ragged=False)
 
     layers = [et.pack_layer(r, cfg.scheme, cfg.ratio, cfg.heads, dtype) for r in raws]
