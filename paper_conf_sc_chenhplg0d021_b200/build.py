@@ -46,12 +46,18 @@ def sources() -> list[str]:
     return sorted(glob.glob(os.path.join(CSRC, "**", "*.cu"), recursive=True))
 
 
-def build(verbose: bool = False, force: bool = False, debug: bool = False) -> str:
-    """Compile every .cu and link libet.so (debug=True: -DET_WATCHDOG build into build/et_dbg/libet_dbg.so)."""
+def build(verbose: bool = False, force: bool = False, debug: bool = False, variant: str | None = None,
+          defines: tuple[str, ...] = ()) -> str:
+    """Compile every .cu and link libet.so (debug=True: -DET_WATCHDOG build into build/et_dbg/libet_dbg.so;
+    variant=NAME: an experiment build with extra -D defines into build/et_var_NAME/libet.so)."""
     nvcc = _nvcc()
-    bdir = BUILD + ("_dbg" if debug else "")
-    lib = os.path.join(bdir, "libet_dbg.so") if debug else LIB
-    flags = FLAGS + (["-DET_WATCHDOG", "-DET_TIMELINE"] if debug else [])
+    if variant:
+        bdir = BUILD + "_var_" + variant
+        lib = os.path.join(bdir, "libet.so")
+    else:
+        bdir = BUILD + ("_dbg" if debug else "")
+        lib = os.path.join(bdir, "libet_dbg.so") if debug else LIB
+    flags = FLAGS + (["-DET_WATCHDOG", "-DET_TIMELINE"] if debug else []) + ["-D" + d for d in defines]
     os.makedirs(bdir, exist_ok=True)
     hdr_mtime = max([os.path.getmtime(h) for h in _headers()] + [0.0])
     jobs = []
@@ -81,4 +87,6 @@ def build(verbose: bool = False, force: bool = False, debug: bool = False) -> st
 
 
 if __name__ == "__main__":
-    print(build(verbose=True, force="--force" in sys.argv, debug="--debug" in sys.argv))
+    var = sys.argv[sys.argv.index("--variant") + 1] if "--variant" in sys.argv else None
+    defs = tuple(a[2:] for a in sys.argv if a.startswith("-D"))
+    print(build(verbose=True, force="--force" in sys.argv, debug="--debug" in sys.argv, variant=var, defines=defs))

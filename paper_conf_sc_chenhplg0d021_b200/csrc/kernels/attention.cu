@@ -101,7 +101,9 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
   constexpr uint32_t kCols = (kO + kDK) <= 256 ? 256u : 512u;
   if (p.v_width && p.v_width[p.head_begin + blockIdx.y] == 0) return;   // every V feature of the head pruned
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-byte aligned, derived from smem_raw by pointer arithmetic so the compiler keeps the shared
+  // address space (an integer round trip would turn every access into a generic LD/ST)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sQ = smem;
   uint8_t* sK = sQ + C::kOpBytes;                // 2 x K block
   uint8_t* sV = sK + 2 * C::kOpBytes;            // 2 x V block

@@ -62,17 +62,33 @@ __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
   float4 part[NP][NCH];
   float4 bias[NCH], res[NCH];
   bool ok[NCH];
+  // Every load is unconditional (out-of-range lanes and absent operands read a valid dummy address
+  // and are masked afterwards): predicated "x = ok ? load : 0" loads make the compiler zero the
+  // destination first and serialise the row's loads behind each other's latency.
+  const bool has_bias = a.bias != nullptr, has_res = a.resid != nullptr;
+  const void* bias_p = has_bias ? a.bias : a.part;
+  const void* res_p = has_res ? a.resid : a.part;
 #pragma unroll
   for (int c = 0; c < NCH; ++c) ok[c] = c * 128 + lane * 4 < a.N;
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
-    const int col = c * 128 + lane * 4;
+    const int col = ok[c] ? c * 128 + lane * 4 : 0;
 #pragma unroll
     for (int q = 0; q < NP; ++q)
-      part[q][c] = ok[c] ? __ldcs(reinterpret_cast<const float4*>(a.part + (size_t)q * a.M * a.N + row + col))
-                         : make_float4(0.f, 0.f, 0.f, 0.f);
-    bias[c] = (ok[c] && a.bias) ? ld_act4<DT>(a.bias, col) : make_float4(0.f, 0.f, 0.f, 0.f);
-    res[c] = (ok[c] && a.resid) ? ld_act4<RT>(a.resid, row + col) : make_float4(0.f, 0.f, 0.f, 0.f);
+      part[q][c] = __ldcs(reinterpret_cast<const float4*>(a.part + (size_t)q * a.M * a.N + row + col));
+    bias[c] = ld_act4<DT>(bias_p, has_bias ? col : 0);
+    res[c] = ld_act4<RT>(res_p, has_res ? row + col : 0);
+  }
+  const float bsc = has_bias ? 1.0f : 0.0f, rsc = has_res ? 1.0f : 0.0f;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const float m = ok[c] ? 1.0f : 0.0f, mb = m * bsc, mr = m * rsc;
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+      part[q][c].x *= m; part[q][c].y *= m; part[q][c].z *= m; part[q][c].w *= m;
+    }
+    bias[c].x *= mb; bias[c].y *= mb; bias[c].z *= mb; bias[c].w *= mb;
+    res[c].x *= mr; res[c].y *= mr; res[c].z *= mr; res[c].w *= mr;
   }
   float4 v[NCH];
   float s = 0.f;

@@ -21,7 +21,9 @@ __global__ void __launch_bounds__(512, 1)
 mma_probe_kernel(const __half* __restrict__ A, const __half* __restrict__ B, float* __restrict__ D, int N,
                  int a_mode, int b_mode, int iters, int n_acc, int issue_mode, long long* __restrict__ cycles) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-byte aligned, derived from smem_raw by pointer arithmetic so the compiler keeps the shared
+  // address space (an integer round trip would turn every access into a generic LD/ST)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sA = smem;                // 16 KB
   uint8_t* sB = smem + 16384;        // up to 32 KB
   __shared__ uint64_t bar;

@@ -4,17 +4,22 @@
 //   Y[m, n] = epilogue( sum over KEPT tiles (i, j) of X[m, 16j:16j+16] . W'[16i:16i+16, 16j:16j+16]^T )
 //
 // One tcgen05.mma (M=128 tokens, N=16 features, K=16) per kept tile; pruned tiles cost nothing.
-// Design (measured in profiles/r01/M1_tcgen05_probe.md):
-//   * the activation block (128 tokens x K<=768) lives in TMEM as the MMA A operand ("TS" MMA):
-//     TMA (SWIZZLE_128B) -> shared memory -> tcgen05.cp.  With A in shared memory every N=16 MMA
-//     re-reads 4 KB of A and the kernel is capped near 20 % of peak by smem bandwidth.
+// Design (measured in profiles/r01/M1_tcgen05_probe.md and profiles/r01/gemm_timeline.md):
+//   * the activation block (128 tokens x K<=768) lives in TMEM as the MMA A operand ("TS" MMA).
+//     With A in shared memory every N=16 MMA re-reads 4 KB of A and the kernel is capped near 20 %
+//     of peak by smem bandwidth.  Fill: TMA (SWIZZLE_128B) -> 3-stage smem ring -> registers of the
+//     16 MMA/epilogue warps (idle during the prologue) -> tcgen05.st; tcgen05.cp moves only ~25 B per
+//     cycle per SM (build with -DET_GEMM_CP_FILL for that path), the register path is TMA-bound.
 //   * packed tiles (512 B each, core-matrix layout) are contiguous per (K part, tile row) and are
 //     streamed with 1-D bulk copies through an 8-stage shared-memory ring.
 //   * 8 MMA warps, one accumulator (16 TMEM columns) each, so 8 independent accumulation chains are
-//     in flight (one warp can only issue an MMA every ~60 cycles; a chain step takes ~110).
-//     Warps 0-3 and 4-7 form two warpgroups working on alternate "quads" of 4 tile rows; a
-//     warpgroup drains its 4 accumulators (tcgen05.ld) while the other one issues MMAs.
-//   * warp 8 fills A (TMA + tcgen05.cp), warp 9 streams the tiles and owns the TMEM allocation.
+//     in flight (one warp can only issue an MMA every ~60 cycles; 8 warps saturate the pipe).  A
+//     warp prepares its next row (barrier waits, tile columns, descriptors) before waiting for its
+//     accumulator to drain, so only the MMA issue sits on the accumulator's critical path.
+//   * two epilogue groups of 4 warps (one per TMEM lane quarter) drain "quads" of 4 accumulators
+//     (64 columns) with one tcgen05.ld, release them, then apply bias / Q-scale / GELU / ReLU in
+//     FP32 (packed FP32x2 arithmetic) and store through 128B-swizzled staging + TMA stores.
+//   * warp 16 issues the A TMA loads, warp 17 streams the tiles and owns the TMEM allocation.
 // Grid: x = piece (a tile-row range of one segment), y = 128-token block, z = K part (split-K,
 // fp32 partial outputs, reduced by the LayerNorm kernel).
 #include <cuda.h>
@@ -32,14 +37,15 @@
 namespace et {
 
 #ifdef ET_TIMELINE
-// Debug builds only: %globaltimer stamps of CTA (0, 0, 0) of the most recent launch.
+// Debug builds only: %clock64 stamps (SM cycles) of CTA (0, 0, 0) of the most recent launch.
 //   slot 0: start; 1: metadata staged; 2..13: A chunk j copied to TMEM (producer); 14: last tile chunk
-//   issued; 16 + 8*w + 2*k, +1: MMA warp w, round k issue start / commit; 96 + 2*r, +1: epilogue row r
-//   accumulator observed / stores issued; 255: end.
+//   issued; 16 + 24*w + 3*k + {0,1,2}: MMA warp w, round k: accumulator free / first MMA / commit;
+//   208 + 40*g + 5*k + {0,1,2,3}: epilogue group g, round k: quad complete / drained / math done /
+//   stores issued; 300: end.
 __device__ unsigned long long g_timeline[512];
 __device__ __forceinline__ unsigned long long gtime() {
   unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
   return t;
 }
 #define ET_TL(slot)                                                              \
@@ -53,8 +59,14 @@ __device__ __forceinline__ unsigned long long gtime() {
 namespace {
 
 constexpr int kMaxPieces = 64;
-constexpr int kNXS = 3;          // X staging stages (16 KB each: 128 rows x 64 K)
-constexpr int kNBS = 8;          // tile staging stages
+#ifndef ET_GEMM_NXS
+#define ET_GEMM_NXS 3
+#endif
+#ifndef ET_GEMM_NBS
+#define ET_GEMM_NBS 8
+#endif
+constexpr int kNXS = ET_GEMM_NXS;   // X staging stages (16 KB each: 128 rows x 64 K)
+constexpr int kNBS = ET_GEMM_NBS;   // tile staging stages
 constexpr int kChunkTiles = 32;  // tiles per stage (16 KB)
 constexpr int kMaxKChunks = 12;  // K <= 768 per part
 constexpr int kMaxBChunks = 192; // tile chunks per CTA (one single-use full barrier each)
@@ -84,6 +96,8 @@ struct Piece {
 struct Params {
   int M, K, Kp, kparts;   // Kp = 768 (K part width); the last part may be shorter
   int box_rows;           // TMA box height: min(128, M) (a box may not exceed the tensor)
+  const uint8_t* X;       // activation block base (K offset k0 folded in)
+  long long ldx_bytes;    // X row pitch in bytes
   int nseg;
   SegDev seg[3];
   int npieces;
@@ -94,10 +108,12 @@ struct Params {
 };
 
 struct __align__(8) Barriers {
-  uint64_t xfull[kNXS], xempty[kNXS], afill[kMaxKChunks];
+  // xfull: one single-use barrier per A chunk (a fill warp may run several ring laps ahead, and a
+  // parity wait on a reused barrier cannot tell those phases apart)
+  uint64_t xfull[kMaxKChunks], xempty[kNXS], afill[kMaxKChunks];
   uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
   uint64_t bfull[kMaxBChunks];
-  int tcol[kNBS][kChunkTiles + 4];   // tile columns of the staged tiles (from a 16-byte aligned start)
+  alignas(16) int tcol[kNBS][kChunkTiles + 4];   // (bulk-copy destination: 16-byte aligned) tile columns of the staged tiles (from a 16-byte aligned start)
   int rptr[kMaxRows + 1];        // this CTA's row pointers, relative to its first tile
   uint32_t bias_s[kMaxRows * 8]; // this CTA's bias slice (16-bit pairs)
   uint32_t tmem_base;
@@ -110,20 +126,26 @@ constexpr size_t kSmemStage = 8 * 4096;   // epilogue staging: 32 rows x 128 B p
 constexpr size_t kSmemBytes = 1024 + kSmemX + kSmemB + kSmemStage + sizeof(Barriers);
 
 // GELU(x) = x Phi(x) = 0.5 x (1 + erf(x / sqrt 2)) (reading C-12), evaluated as
-//   0.5 erfc(t) = 2^(-g(t) - 1),  t = |x| / sqrt 2 clamped to 4,  g(t) = -log2 erfc(t) ~ t q(t)
-// with q a degree-5 polynomial fitted on [0, 4] (tools/fit_gelu.py): |GELU error| <= 6.3e-7 in FP32
-// (below FP16/BF16 output resolution) for ~12 instructions and one ex2, half the cost of erff().
-__device__ __forceinline__ float gelu_erf(float x) {
-  const float t = fminf(fabsf(x) * 0.70710678118654752f, 4.0f);
-  float q = -0.00015888f;
-  q = fmaf(q, t, 0.0037465857f);
-  q = fmaf(q, t, -0.0310388145f);
-  q = fmaf(q, t, 0.1498060619f);
-  q = fmaf(q, t, 0.9181324485f);
-  q = fmaf(q, t, 1.6279282351f);
-  float e;   // 0.5 * erfc(t)
-  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e) : "f"(-fmaf(t, q, 1.0f)));
-  return x * (x >= 0.f ? 1.0f - e : e);
+//   GELU(x) = max(x, 0) - |x| e,   e = 0.5 erfc(t) = 2^(-g(t) - 1),   t = |x| / sqrt 2 (clamped to 4)
+// (x >= 0: x (1 - e); x < 0: x e), with g(t) = -log2 erfc(t) ~ t q(t), q a degree-5 polynomial fitted
+// on [0, 4] (tools/fit_gelu.py): |GELU error| <= 6.3e-7 in FP32, below FP16/BF16 output resolution.
+// Two elements at a time with packed FP32x2 FMAs: 16 instructions (two MUFU.EX2) per pair.  The
+// factor sqrt 2 of -|x| e = (-t)(sqrt 2 e) is folded into the exponent (-t q - 1/2).
+__device__ __forceinline__ void gelu_erf2(float& x0, float& x1) {
+  const float tn0 = fabsf(x0) * -0.70710678118654752f, tn1 = fabsf(x1) * -0.70710678118654752f;
+  const uint64_t t = f2pk(fminf(-tn0, 4.0f), fminf(-tn1, 4.0f));
+  uint64_t q = ffma2(f2pk(0.00015888f, 0.00015888f), t, f2pk(-0.0037465857f, -0.0037465857f));   // -q(t)
+  q = ffma2(q, t, f2pk(0.0310388145f, 0.0310388145f));
+  q = ffma2(q, t, f2pk(-0.1498060619f, -0.1498060619f));
+  q = ffma2(q, t, f2pk(-0.9181324485f, -0.9181324485f));
+  q = ffma2(q, t, f2pk(-1.6279282351f, -1.6279282351f));
+  const float2 y = f2upk(ffma2(t, q, f2pk(-0.5f, -0.5f)));   // -t q(t) - 1/2
+  float e0, e1;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e0) : "f"(y.x));
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e1) : "f"(y.y));
+  const float2 g = f2upk(ffma2(f2pk(tn0, tn1), f2pk(e0, e1), f2pk(fmaxf(x0, 0.0f), fmaxf(x1, 0.0f))));
+  x0 = g.x;
+  x1 = g.y;
 }
 
 template <int kEpi, bool kBF16>
@@ -131,7 +153,9 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
                                                              const __grid_constant__ CUtensorMap tmap_y,
                                                              const __grid_constant__ Params p) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-byte aligned, derived from smem_raw by pointer arithmetic so the compiler keeps the shared
+  // address space (an integer round trip would turn every access into a generic LD/ST)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sX = smem;
   uint8_t* sB = smem + kSmemX;
   uint8_t* sStage = smem + kSmemX + kSmemB;
@@ -153,11 +177,18 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
   if (threadIdx.x == 0) ET_TL(0);
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kNXS; ++i) {
-      mbar_init(&bar.xfull[i], 1);
-      mbar_init(&bar.xempty[i], 1);
-    }
+#ifndef ET_GEMM_CP_FILL
+    constexpr int kFillArrivals = 4;   // four register-fill warps per chunk
+#else
+    constexpr int kFillArrivals = 1;   // one tcgen05.commit per chunk
+#endif
+    for (int i = 0; i < kNXS; ++i) mbar_init(&bar.xempty[i], kFillArrivals);
+    for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.xfull[i], 1);
+#ifndef ET_GEMM_CP_FILL
+    for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.afill[i], kFillArrivals);
+#else
     for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.afill[i], 1);
+#endif
     for (int i = 0; i < kMmaWarps; ++i) {
       mbar_init(&bar.acc_full[i], 1);
       mbar_init(&bar.acc_empty[i], 4);
@@ -183,6 +214,39 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const uint32_t tbase = bar.tmem_base;
   if (threadIdx.x == 0) ET_TL(1);
 
+#ifndef ET_GEMM_CP_FILL
+  if (warp < 16) {
+    // smem ring -> TMEM through registers (instead of tcgen05.cp): chunk j is moved by the four
+    // warps with w / 4 == j % 4, warp w taking TMEM lane quarter w % 4 (its 32 token rows); lane i
+    // reads its row's 128 bytes from the SWIZZLE_128B chunk (16-byte unit c of row r sits at unit
+    // c ^ (r % 8): conflict-free) and one tcgen05.st.32x32b.x32 writes 32 packed columns.
+    const int q = warp & 3;
+    const int rr = q * 32 + lane;
+    const uint32_t tq = tbase + ((uint32_t)(q * 32) << 16);
+#pragma unroll 1
+    for (int j = warp >> 2; j < nk; j += 4) {
+      const int slot = j % kNXS;
+      mbar_wait_warp(&bar.xfull[j], 0);
+      const uint8_t* rowp = sX + slot * 16384 + rr * 128;
+      uint32_t v[32];
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        const uint4 u = *reinterpret_cast<const uint4*>(rowp + ((c ^ (rr & 7)) << 4));
+        v[4 * c] = u.x; v[4 * c + 1] = u.y; v[4 * c + 2] = u.z; v[4 * c + 3] = u.w;
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&bar.xempty[slot]);   // the TMA thread may refill the slot
+      tmem_st32(tq + j * 32, v);
+      tmem_st_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&bar.afill[j]);
+    }
+  }
+  if (warp == kWarpCp) {
+    // idle in this build
+  } else
+#endif
   if (warp == kWarpA) {
     // ===================== A producer (TMA): X block -> smem ring, up to kNXS chunks ahead
     if (lane == 0) {
@@ -191,8 +255,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       for (int j = 0; j < nk; ++j) {
         const int slot = j % kNXS;
         if (j >= kNXS) mbar_wait(&bar.xempty[slot], ((j / kNXS) - 1) & 1);
-        mbar_expect_tx(&bar.xfull[slot], p.box_rows * 128);
-        tma_load_2d(sX + slot * 16384, &tmap_x, &bar.xfull[slot], kx0 + j * 64, m0);
+        mbar_expect_tx(&bar.xfull[j], p.box_rows * 128);
+        tma_load_2d(sX + slot * 16384, &tmap_x, &bar.xfull[j], kx0 + j * 64, m0);
       }
     }
   } else if (warp == kWarpCp) {
@@ -200,7 +264,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     if (lane == 0) {
       for (int j = 0; j < nk; ++j) {
         const int slot = j % kNXS;
-        mbar_wait(&bar.xfull[slot], (j / kNXS) & 1);
+        mbar_wait(&bar.xfull[j], 0);
         tc_fence_after();
         const uint32_t src = smem_u32(sX + slot * 16384);
 #pragma unroll
@@ -223,8 +287,15 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     if (lane == 0) {
       const uint8_t* vals = sg.values + (size_t)pb * 512;
       int tl = 0;   // last local row that starts before the end of the chunk being recycled
+      // Chunks beyond what round 0 needs wait until the A block is in TMEM: in the prologue every
+      // CTA of the grid streams its A block at once and the chip's L2 bandwidth is the limit, so
+      // tile prefetch would only delay the first MMAs.
+      const int c_r0 = (bar.rptr[min(kMmaWarps, nrows)] + kChunkTiles - 1) / kChunkTiles + 1;
       for (int c = 0; c < nchunks; ++c) {
         const int slot = c % kNBS;
+#ifndef ET_GEMM_EAGER_B
+        if (c == c_r0) mbar_wait(&bar.afill[nk - 1], 0);
+#endif
         if (c >= kNBS) {
           const int end_tile = pb + (c - kNBS + 1) * kChunkTiles;
           while (tl + 1 < nrows && bar.rptr[tl + 1] + pb < end_tile) ++tl;
@@ -256,17 +327,16 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     for (int k = 0; k < nrounds; ++k) {
       const int t = k * kMmaWarps + warp;
       if (t >= nrows) break;
-      if (k > 0) {   // the epilogue group must have read this accumulator's previous row
-        mbar_wait_warp(&bar.acc_empty[warp], (k - 1) & 1);
-        tc_fence_after();
-      }
-      if (lane == 0) ET_TL(16 + 8 * warp + 2 * k);
       const int q0 = bar.rptr[t], q1 = bar.rptr[t + 1];   // this row's tiles, relative to pb
-      // the row's tiles lie in chunks [q0 / 32, (q1 - 1) / 32]: wait for each once, then read the
-      // tile columns lane-parallel and issue the MMAs from register broadcasts
-      for (int qb = q0; qb < q1;) {
+      // The row's tiles lie in chunks [q0 / 32, (q1 - 1) / 32].  A segment = the row's tiles inside
+      // one chunk: wait for the chunk once, read the tile columns lane-parallel, issue the MMAs from
+      // register broadcasts.  The first segment is prepared BEFORE waiting for the accumulator, so
+      // the barrier / shared-memory / shuffle latency stays off the accumulator's critical path.
+      int qb = q0, qe = q0, n = 0;
+      uint32_t acol = 0, blo = 0, bhi = 0;
+      auto prep = [&]() {
         const int c = qb / kChunkTiles;
-        const int qe = min(q1, (c + 1) * kChunkTiles);   // tiles of this row inside chunk c
+        qe = min(q1, (c + 1) * kChunkTiles);
         if (c != cur_chunk) {
           mbar_wait_warp(&bar.bfull[c], 0);
           cur_chunk = c;
@@ -274,24 +344,32 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         }
         const int slot = c % kNBS;
         const int coff = (pb + c * kChunkTiles) & 3;
-        const int n = qe - qb;
+        n = qe - qb;
         const int mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
         int maxcol = mycol;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) maxcol = max(maxcol, __shfl_xor_sync(0xffffffffu, maxcol, o));
-        if ((maxcol >> 2) > a_ready) {   // all A chunks this segment needs (afill[j] implies all < j)
-          mbar_wait_warp(&bar.afill[maxcol >> 2], 0);
-          a_ready = maxcol >> 2;
+        if ((maxcol >> 2) > a_ready) {   // every A chunk up to the segment's last tile column
+          while (a_ready < (maxcol >> 2)) mbar_wait_warp(&bar.afill[++a_ready], 0);
           tc_fence_after();
         }
         // B descriptor of tile u: start address field advances by 512 B / 16 = 32 per tile
         const uint64_t bd0 = make_sdesc(sB_u32 + slot * (kChunkTiles * 512) + (qb % kChunkTiles) * 512, 128, 256,
                                         kLayoutNone);
-        const uint32_t blo = (uint32_t)bd0, bhi = (uint32_t)(bd0 >> 32);
-        const uint32_t acol = tbase + (uint32_t)(mycol * 8);   // this lane's tile: its A columns
+        blo = (uint32_t)bd0;
+        bhi = (uint32_t)(bd0 >> 32);
+        acol = tbase + (uint32_t)(mycol * 8);   // this lane's tile: its A columns
+      };
+      if (qb < q1) prep();
+      if (k > 0) {   // the epilogue group must have read this accumulator's previous row
+        mbar_wait_warp(&bar.acc_empty[warp], (k - 1) & 1);
+        tc_fence_after();
+      }
+      if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k);
+      while (qb < q1) {
         int u = 0;
         for (; u + 4 <= n; u += 4) {
-          if (warp == 0 && k == 1 && lane == 0 && qb + u - q0 < 24) ET_TL(300 + (qb + u - q0));
+          if (lane == 0 && k < 8 && qb + u == q0) ET_TL(16 + 24 * warp + 3 * k + 1);
           mma_ts_warp_x4(d_tmem, __shfl_sync(0xffffffffu, acol, u), __shfl_sync(0xffffffffu, acol, u + 1),
                          __shfl_sync(0xffffffffu, acol, u + 2), __shfl_sync(0xffffffffu, acol, u + 3),
                          blo + 32 * u, blo + 32 * (u + 1), blo + 32 * (u + 2), blo + 32 * (u + 3), bhi, idesc,
@@ -302,9 +380,10 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           mma_ts_warp_nc(d_tmem, a, ((uint64_t)bhi << 32) | (blo + 32 * u), idesc, (qb + u) != q0);
         }
         qb = qe;
+        if (qb < q1) prep();
       }
       mma_commit_warp(&bar.acc_full[warp]);   // fires when this row's MMAs are complete
-      if (lane == 0) ET_TL(16 + 8 * warp + 2 * k + 1);
+      if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k + 2);
     }
   } else {
     // ===================== epilogue warps: group g drains the accumulators of MMA warps 4g..4g+3
@@ -317,14 +396,14 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       const int t0 = k * kMmaWarps + g * 4;   // first row of this group's quad in round k
       if (t0 >= nrows) break;
       const int na = min(4, nrows - t0);
+      uint32_t r[64];
       for (int a = 0; a < na; ++a) {
         mbar_wait_warp(&bar.acc_full[g * 4 + a], k & 1);
-        if (k == 1 && g == 0 && a == 0 && quarter == 0 && lane == 0) ET_TL(330);
       }
+      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k);
       tc_fence_after();
       if (quarter == 0 && lane == 0)
         st_release_shared(&bar.rows_seen[g], k * 4 + na);   // rows' MMAs complete: their B tiles are free
-      uint32_t r[64];
       tmem_ld32(tbase + kAccCol + g * 64 + ((uint32_t)(quarter * 32) << 16), *reinterpret_cast<uint32_t(*)[32]>(r));
       tmem_ld32(tbase + kAccCol + g * 64 + 32 + ((uint32_t)(quarter * 32) << 16),
                 *reinterpret_cast<uint32_t(*)[32]>(r + 32));
@@ -333,38 +412,39 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       __syncwarp();
       if (lane == 0)
         for (int a = 0; a < na; ++a) mbar_arrive(&bar.acc_empty[g * 4 + a]);
-      if (quarter == 0 && lane == 0) ET_TL(96 + 2 * t0);
+      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 1);
       // math: bias / scale / activation on the quad's 64 columns of this thread's token row
       float v[64];
 #pragma unroll
       for (int a = 0; a < 4; ++a) {
         const int t = t0 + min(a, na - 1);
-        const bool empty_row = a >= na || bar.rptr[t + 1] == bar.rptr[t];   // never written: zero
-        float b[16];
-        if constexpr (kEpi != ET_EPI_F32) {
+        const bool empty_row = a >= na || bar.rptr[t + 1] == bar.rptr[t];
 #pragma unroll
-          for (int c = 0; c < 8; ++c) {
-            const float2 f = unpack2<kBF16>(bar.bias_s[t * 8 + c]);
-            b[2 * c] = f.x;
-            b[2 * c + 1] = f.y;
-          }
-        }
-#pragma unroll
-        for (int c = 0; c < 16; ++c) {
-          float x = empty_row ? 0.f : __uint_as_float(r[a * 16 + c]);
+        for (int c = 0; c < 16; c += 2) {
+          // a row with no kept tile was never written: its accumulator is zero (output = epi(bias))
+          float x0 = empty_row ? 0.0f : __uint_as_float(r[a * 16 + c]);
+          float x1 = empty_row ? 0.0f : __uint_as_float(r[a * 16 + c + 1]);
           if constexpr (kEpi != ET_EPI_F32) {
-            x += b[c];
+            const float2 bb = unpack2<kBF16>(bar.bias_s[t * 8 + c / 2]);
+            uint64_t xx = fadd2(f2pk(x0, x1), f2pk(bb.x, bb.y));
             if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
-              if (sg.apply_scale) x *= sg.scale;
-            } else if constexpr (kEpi == ET_EPI_BIAS_GELU) {
-              x = gelu_erf(x);
+              if (sg.apply_scale) xx = fmul2(xx, f2pk(sg.scale, sg.scale));
+            }
+            const float2 xf = f2upk(xx);
+            x0 = xf.x;
+            x1 = xf.y;
+            if constexpr (kEpi == ET_EPI_BIAS_GELU) {
+              gelu_erf2(x0, x1);
             } else if constexpr (kEpi == ET_EPI_BIAS_RELU) {
-              x = fmaxf(x, 0.0f);
+              x0 = fmaxf(x0, 0.0f);
+              x1 = fmaxf(x1, 0.0f);
             }
           }
-          v[a * 16 + c] = x;
+          v[a * 16 + c] = x0;
+          v[a * 16 + c + 1] = x1;
         }
       }
+      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 2);
       // store: registers -> this warp's 32-row staging tile (128 B rows, SWIZZLE_128B, conflict-free)
       // -> one TMA tensor store per 128-byte column block (clipped at M by the tensor map)
       uint8_t* st = sStage + (warp - kMmaWarps) * 4096;
@@ -421,7 +501,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           }
         }
       }
-      if (quarter == 0 && lane == 0) ET_TL(96 + 2 * t0 + 1);
+      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 3);
     }
   }
 
@@ -429,7 +509,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   __syncwarp();   // producer warps: lane 0 ran the loops alone; reconverge before the block barrier
   tc_fence_before();
   __syncthreads();
-  if (threadIdx.x == 0) ET_TL(255);
+  if (threadIdx.x == 0) ET_TL(300);
   if (warp == kWarpB) {
     __syncwarp();
     tc_fence_after();
@@ -535,6 +615,8 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   prm.M = a.M;
   prm.K = a.K;
   prm.box_rows = a.M < 128 ? a.M : 128;
+  prm.X = static_cast<const uint8_t*>(a.X) + (size_t)a.k0 * 2;
+  prm.ldx_bytes = (long long)a.ldx * 2;
   prm.Kp = kparts > 1 ? 768 : a.K;
   prm.kparts = kparts;
   prm.nseg = a.nseg;

@@ -1,0 +1,15 @@
+#!/bin/bash
+# Run on the GPU box (gpurun): launch list of the bench command + one --set full capture per kernel
+# kind of the C3 encoder's second call (layer 0).  Output under gpurun_out/.
+set -x
+mkdir -p gpurun_out
+ncu --metrics gpu__time_duration.sum --clock-control none -c 2500 --csv --log-file gpurun_out/launches.csv \
+    python bench.py --steps 2 --warmup 3 > gpurun_out/launches_bench.log 2>&1
+# 84 launches per encoder call; skip the first call
+ncu --set full --clock-control none --import-source on -k regex:tsgemm -s 48 -c 4 -f -o gpurun_out/prof_gemm \
+    python tools/prof_layer.py > gpurun_out/prof_gemm.log 2>&1
+ncu --set full --clock-control none --import-source on -k regex:attn_kernel -s 12 -c 1 -f -o gpurun_out/prof_attn \
+    python tools/prof_layer.py > gpurun_out/prof_attn.log 2>&1
+ncu --set full --clock-control none --import-source on -k regex:layernorm -s 24 -c 2 -f -o gpurun_out/prof_ln \
+    python tools/prof_layer.py > gpurun_out/prof_ln.log 2>&1
+ls -la gpurun_out
