@@ -39,7 +39,7 @@ class EtError(RuntimeError):
 
 def _load():
     if not os.path.exists(LIB_PATH):
-        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_sc_chenhplg0d021_b200.build` "
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python paper_conf_sc_chenhplg0d021_b200/build.py` "
                           "(there is no CPU fallback)")
     return ctypes.CDLL(LIB_PATH)
 

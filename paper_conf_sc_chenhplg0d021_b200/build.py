@@ -1,6 +1,6 @@
 """Build libet.so (the C-ABI library) in-tree for sm_100a.
 
-    python -m paper_conf_sc_chenhplg0d021_b200.build      (or __graft_entry__.build())
+    python paper_conf_sc_chenhplg0d021_b200/build.py      (or __graft_entry__.build())
 
 Every .cu under csrc/ is compiled with
     nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -lineinfo -Xcompiler -fPIC
