@@ -93,8 +93,16 @@ class ClockSampler:
             h = None
             try:
                 import torch
-                bus = torch.cuda.get_device_properties(gpu_index).pci_bus_id
-                h = pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+                # torch's pci_* properties are integers: match them against every NVML device
+                pr = torch.cuda.get_device_properties(gpu_index)
+                for i in range(pynvml.nvmlDeviceGetCount()):
+                    hi = pynvml.nvmlDeviceGetHandleByIndex(i)
+                    pci = pynvml.nvmlDeviceGetPciInfo(hi)
+                    if (pci.bus, pci.device, pci.domain) == (pr.pci_bus_id, pr.pci_device_id, pr.pci_domain_id):
+                        h = hi
+                        break
+                if h is None:
+                    raise RuntimeError("no NVML device matches the CUDA device")
             except Exception:
                 h = pynvml.nvmlDeviceGetHandleByIndex(gpu_index)
             self.nvml, self.h = pynvml, h
