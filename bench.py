@@ -317,68 +317,82 @@ def our_arm(args):
         if dist is not None:
             dist.barrier()
 
-    for _ in range(max(args.warmup, 3)):
+    for _ in range(3):   # eager calls: first-use kernel attributes, tensor-map encoder
         enc(Xd, out)
     torch.cuda.synchronize()
-
-    # ---------------- timed region: K steps, per-step events, L2 flushed between steps
+    # the forward as one CUDA graph (et_encoder_graph_create): the timed unit is one replay
+    graph = enc.capture(Xd, out)
     K = args.steps
-    cap = K * (len(layers) * 8 + 4) + 8
+    cap = len(layers) * 8 + 4
+    et._check(et._lib.et_trace_begin(cap))
+    graph_tr = enc.capture(Xd, out)       # same kernels + external event-record nodes per kernel
+    n_int = __import__("ctypes").c_int32()
+    et._check(et._lib.et_trace_end(__import__("ctypes").byref(n_int)))
+    for _ in range(max(args.warmup, 3)):
+        graph.launch()
+    torch.cuda.synchronize()
+
+    # ---------------- timed region: K steps (graph replays), per-step events, L2 flushed between steps
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
     clk = ClockSampler(local)
     barrier()
     torch.cuda.synchronize()
     clk.start()
     launches0 = et._lib.et_launch_count()
-    et._check(et._lib.et_trace_begin(cap))
     for s in range(K):
         flush.fill_(float(s))
         ev[s][0].record(stream)
-        enc(Xd, out)
+        graph.launch()
         ev[s][1].record(stream)
-    n_int = __import__("ctypes").c_int32()
-    et._check(et._lib.et_trace_end(__import__("ctypes").byref(n_int)))
     launches = et._lib.et_launch_count() - launches0
     torch.cuda.synchronize()
     barrier()
     clocks = clk.stop()
     step_ms = [a.elapsed_time(b) for a, b in ev]
     t_local = sum(step_ms) / 1e3
-    # per-kernel trace
+
+    # ---------------- per-kernel device time: K replays of the traced graph, same flush discipline
     import ctypes
     kind = ctypes.c_int32()
     ms = ctypes.c_float()
     per_kind = {}
-    for i in range(n_int.value):
-        et._check(et._lib.et_trace_get(i, ctypes.byref(kind), ctypes.byref(ms)))
-        if kind.value < len(KIND_NAMES):
-            per_kind.setdefault(KIND_NAMES[kind.value], []).append(ms.value)
+    tr_ms = []
+    for s in range(K):
+        flush.fill_(float(s))
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        graph_tr.launch()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        tr_ms.append(e0.elapsed_time(e1))
+        for i in range(n_int.value):
+            et._check(et._lib.et_trace_get(i, ctypes.byref(kind), ctypes.byref(ms)))
+            if kind.value < len(KIND_NAMES):
+                per_kind.setdefault(KIND_NAMES[kind.value], []).append(ms.value)
 
-    # ---------------- end to end: pinned host input -> device, forward, device -> pinned host output
+    # ---------------- end to end: pinned host input -> device, graph replay, device -> pinned host output
     e2e = None
     if not args.no_e2e:
         Xh = torch.from_numpy(np.ascontiguousarray(X.reshape(cfg.tokens, cfg.d_model))).to(tdt).pin_memory()
         Oh = torch.empty_like(Xh).pin_memory()
-        Xin = torch.empty_like(Xd)
         eev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
         for _ in range(2):
-            Xin.copy_(Xh, non_blocking=True)
-            enc(Xin, out)
+            Xd.copy_(Xh, non_blocking=True)
+            graph.launch()
             Oh.copy_(out, non_blocking=True)
         torch.cuda.synchronize()
         barrier()
         for s in range(K):
             flush.fill_(float(s))
             eev[s][0].record(stream)
-            Xin.copy_(Xh, non_blocking=True)
-            enc(Xin, out)
+            Xd.copy_(Xh, non_blocking=True)
+            graph.launch()
             Oh.copy_(out, non_blocking=True)
             eev[s][1].record(stream)
         torch.cuda.synchronize()
         barrier()
         e2e_local = sum(a.elapsed_time(b) for a, b in eev) / 1e3
-        e2e = {"t": e2e_local, "h2d": Xh.numel() * Xh.element_size() + L.numel() * 0,
-               "d2h": Oh.numel() * Oh.element_size()}
+        e2e = {"t": e2e_local, "h2d": Xh.numel() * Xh.element_size(), "d2h": Oh.numel() * Oh.element_size()}
 
     # ---------------- max over ranks
     t_max = t_local
@@ -441,6 +455,8 @@ def our_arm(args):
             "gpu_launches": int(launches),
             "clocks": clocks,
             "step_ms_p50": statistics.median(step_ms),
+            "traced_step_ms_p50": statistics.median(tr_ms),
+            "launch": "one CUDA graph replay per step (et_encoder_graph_create / et_graph_launch)",
         }
         if e2e:
             line["e2e"] = {"value": total_seqs / e2e_max, "unit": "seqs/s", "h2d_bytes_per_step": e2e["h2d"],

@@ -221,6 +221,26 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
                          et_dtype resid_dtype, const et_layer* layers_host, const void* X, void* out,
                          void* workspace, size_t ws_bytes, void* stream);
 
+/* CUDA-graph plan of one et_encoder_fwd call (the paper's model is a fixed stack of layers run
+ * again and again on new inputs of the same shape): the whole forward
+ * (12 layers x 7 kernels for BERT-base) is captured once and replayed with one launch, removing
+ * the host-side launch cost that otherwise exceeds the device time at small batches.
+ *   et_encoder_graph_create: same arguments as et_encoder_fwd; captures on a private stream
+ *     (thread-local capture mode) and instantiates.  Every pointer (X, out, workspace, the layers'
+ *     device buffers, desc->lengths_dev) is baked into the graph: later launches read and write
+ *     the same addresses, so the caller keeps them alive and refills X in place.  If tracing is
+ *     enabled (et_trace_begin) during creation, the trace events are captured too and every
+ *     launch re-records them (et_trace_get then reports the most recent launch).
+ *   et_graph_launch: enqueue one replay on `stream`.
+ *   et_graph_destroy: free the host-side graph objects (NULL is allowed).
+ * Errors: the et_encoder_fwd validation errors; ET_ERR_CUDA if capture or instantiation fails. */
+typedef struct et_graph et_graph;
+et_status et_encoder_graph_create(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff, et_act act,
+                                  float ln_eps, et_dtype resid_dtype, const et_layer* layers_host, const void* X,
+                                  void* out, void* workspace, size_t ws_bytes, et_graph** graph);
+et_status et_graph_launch(et_graph* graph, void* stream);
+et_status et_graph_destroy(et_graph* graph);
+
 /* ------------------------------------------------------------------------------------------
  * Tracing (calling thread only): while enabled, the forward entry points record a CUDA event on
  * the caller's stream before every kernel they launch (and one after the last), tagged with the

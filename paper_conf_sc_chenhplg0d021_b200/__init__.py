@@ -248,6 +248,13 @@ _enc = _sig("et_encoder_fwd", ctypes.c_int,
             [ctypes.POINTER(AttnDescC), _i32, _i32, ctypes.c_int, _f32, ctypes.c_int, ctypes.POINTER(LayerC), _vp,
              _vp, _vp, _sz, _vp])
 
+_graph_create = _sig("et_encoder_graph_create", ctypes.c_int,
+                     [ctypes.POINTER(AttnDescC), _i32, _i32, ctypes.c_int, _f32, ctypes.c_int, ctypes.POINTER(LayerC),
+                      _vp, _vp, _vp, _sz, ctypes.POINTER(ctypes.c_void_p)])
+_graph_launch = _sig("et_graph_launch", ctypes.c_int, [ctypes.c_void_p, _vp])
+_graph_destroy = _sig("et_graph_destroy", ctypes.c_int, [ctypes.c_void_p])
+SYMBOLS += ["et_encoder_graph_create", "et_graph_launch", "et_graph_destroy"]
+
 
 def attn_desc(batch, seq_len, heads, d_model, dtype, lengths=None, causal=False, mode="auto",
               head_begin=0, head_end=None) -> AttnDescC:
@@ -361,6 +368,32 @@ class Encoder:
         _check(_enc(ctypes.byref(self.desc), len(self.layers), self.d_ff, self.act, self.eps, self.resid_dtype,
                     self.arr, X.data_ptr(), out.data_ptr(), self.ws.data_ptr(), self.ws.numel(), _stream(stream)))
         return out
+
+
+    def capture(self, X: torch.Tensor, out: torch.Tensor) -> "Graph":
+        """et_encoder_graph_create: the whole forward on (X, out) as one CUDA graph (X is read in place
+        at every launch; X, out, the workspace and the layers must outlive the graph)."""
+        g = ctypes.c_void_p()
+        _check(_graph_create(ctypes.byref(self.desc), len(self.layers), self.d_ff, self.act, self.eps,
+                             self.resid_dtype, self.arr, X.data_ptr(), out.data_ptr(), self.ws.data_ptr(),
+                             self.ws.numel(), ctypes.byref(g)))
+        return Graph(g, keep=(self, X, out))
+
+
+class Graph:
+    """A captured forward (et_graph*): launch() enqueues one replay on the current stream."""
+
+    def __init__(self, handle: ctypes.c_void_p, keep=()):
+        self.h = handle
+        self._keep = keep
+
+    def launch(self, stream=None):
+        _check(_graph_launch(self.h, _stream(stream)))
+
+    def __del__(self):
+        if getattr(self, "h", None) is not None and self.h.value:
+            _graph_destroy(self.h)
+            self.h = None
 
 
 def encoder_fwd(X: torch.Tensor, layers: list, batch: int, seq_len: int, heads: int, d_ff: int, **kw):

@@ -43,6 +43,8 @@ static thread_local Trace g_trace;
 static thread_local long long g_launches = 0;
 
 void count_launch() { ++g_launches; }
+void add_launches(long long n) { g_launches += n; }
+long long launch_count() { return g_launches; }
 
 void trace_mark(int kind, cudaStream_t stream) {
   Trace& t = g_trace;
@@ -53,7 +55,12 @@ void trace_mark(int kind, cudaStream_t stream) {
     t.ev.push_back(e);
     t.kind.push_back(0);
   }
-  cudaEventRecord(t.ev[t.n], stream);
+  // inside a stream capture the event must be an external record node so that every replay of
+  // the graph records it again (a plain record would only order the capture)
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaStreamIsCapturing(stream, &cs);
+  if (cs == cudaStreamCaptureStatusActive) cudaEventRecordWithFlags(t.ev[t.n], stream, cudaEventRecordExternal);
+  else cudaEventRecord(t.ev[t.n], stream);
   t.kind[t.n] = kind;
   ++t.n;
 }

@@ -392,4 +392,58 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
   return ET_OK;
 }
 
+struct et_graph {
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  long long kernels = 0;   // library kernels per replay (launch accounting)
+};
+
+et_status et_encoder_graph_create(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff, et_act act,
+                                  float ln_eps, et_dtype resid_dtype, const et_layer* layers, const void* X,
+                                  void* out, void* workspace, size_t ws_bytes, et_graph** graph) {
+  if (!graph) return fail(ET_ERR_INVALID_ARG, "et_encoder_graph_create: null graph pointer");
+  *graph = nullptr;
+  cudaStream_t cs = nullptr;
+  ET_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  et_graph* g = new et_graph();
+  const long long l0 = launch_count();
+  cudaError_t e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
+  et_status st = e == cudaSuccess ? ET_OK : fail(ET_ERR_CUDA, "cudaStreamBeginCapture: %s", cudaGetErrorString(e));
+  if (st == ET_OK) {
+    st = et_encoder_fwd(desc, num_layers, d_ff, act, ln_eps, resid_dtype, layers, X, out, workspace, ws_bytes, cs);
+    cudaGraph_t gr = nullptr;
+    e = cudaStreamEndCapture(cs, &gr);   // always end the capture, even after a failed forward
+    if (st == ET_OK && e != cudaSuccess) st = fail(ET_ERR_CUDA, "cudaStreamEndCapture: %s", cudaGetErrorString(e));
+    g->graph = gr;
+  }
+  if (st == ET_OK) {
+    e = cudaGraphInstantiate(&g->exec, g->graph, 0);
+    if (e != cudaSuccess) st = fail(ET_ERR_CUDA, "cudaGraphInstantiate: %s", cudaGetErrorString(e));
+  }
+  g->kernels = launch_count() - l0;
+  add_launches(-g->kernels);   // nothing ran yet: the kernels are counted when the graph launches
+  cudaStreamDestroy(cs);
+  if (st != ET_OK) {
+    et_graph_destroy(g);
+    return st;
+  }
+  *graph = g;
+  return ET_OK;
+}
+
+et_status et_graph_launch(et_graph* g, void* stream) {
+  if (!g || !g->exec) return fail(ET_ERR_INVALID_ARG, "et_graph_launch: null graph");
+  ET_CUDA(cudaGraphLaunch(g->exec, static_cast<cudaStream_t>(stream)));
+  add_launches(g->kernels);
+  return ET_OK;
+}
+
+et_status et_graph_destroy(et_graph* g) {
+  if (!g) return ET_OK;
+  if (g->exec) cudaGraphExecDestroy(g->exec);
+  if (g->graph) cudaGraphDestroy(g->graph);
+  delete g;
+  return ET_OK;
+}
+
 }  // extern "C"

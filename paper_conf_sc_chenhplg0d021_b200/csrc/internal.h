@@ -130,5 +130,7 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream);
 // Record a mark of `kind` on `stream` if tracing is enabled; counts one kernel launch.
 void trace_mark(int kind, cudaStream_t stream);
 void count_launch();
+void add_launches(long long n);
+long long launch_count();
 
 }  // namespace et

@@ -4,22 +4,23 @@
 //   Y[m, n] = epilogue( sum over KEPT tiles (i, j) of X[m, 16j:16j+16] . W'[16i:16i+16, 16j:16j+16]^T )
 //
 // One tcgen05.mma (M=128 tokens, N=16 features, K=16) per kept tile; pruned tiles cost nothing.
-// Design (measured in profiles/r01/M1_tcgen05_probe.md and profiles/r01/gemm_timeline.md):
+// Design (measured in profiles/r01/M1_tcgen05_probe.md and the cycle timelines of profiles/r01):
 //   * the activation block (128 tokens x K<=768) lives in TMEM as the MMA A operand ("TS" MMA).
 //     With A in shared memory every N=16 MMA re-reads 4 KB of A and the kernel is capped near 20 %
-//     of peak by smem bandwidth.  Fill: TMA (SWIZZLE_128B) -> 3-stage smem ring -> registers of the
-//     16 MMA/epilogue warps (idle during the prologue) -> tcgen05.st; tcgen05.cp moves only ~25 B per
-//     cycle per SM (build with -DET_GEMM_CP_FILL for that path), the register path is TMA-bound.
-//   * packed tiles (512 B each, core-matrix layout) are contiguous per (K part, tile row) and are
-//     streamed with 1-D bulk copies through an 8-stage shared-memory ring.
+//     of peak by smem bandwidth.  Fill: TMA (SWIZZLE_128B) -> smem -> registers of the 24 MMA /
+//     epilogue warps (idle during the prologue) -> tcgen05.st.
+//   * one unified 9-slot shared-memory ring carries first the A chunks (all in flight at once: the
+//     prologue is bound by L2 bandwidth, not by ring depth) and then the packed tiles (512 B each,
+//     contiguous per (K part, tile row), 1-D bulk copies of 32 tiles + their column indices).
 //   * 8 MMA warps, one accumulator (16 TMEM columns) each, so 8 independent accumulation chains are
 //     in flight (one warp can only issue an MMA every ~60 cycles; 8 warps saturate the pipe).  A
 //     warp prepares its next row (barrier waits, tile columns, descriptors) before waiting for its
 //     accumulator to drain, so only the MMA issue sits on the accumulator's critical path.
-//   * two epilogue groups of 4 warps (one per TMEM lane quarter) drain "quads" of 4 accumulators
-//     (64 columns) with one tcgen05.ld, release them, then apply bias / Q-scale / GELU / ReLU in
-//     FP32 (packed FP32x2 arithmetic) and store through 128B-swizzled staging + TMA stores.
-//   * warp 16 issues the A TMA loads, warp 17 streams the tiles and owns the TMEM allocation.
+//   * four epilogue groups of 4 warps (one per TMEM lane quarter) each drain a pair of accumulators
+//     (32 columns) with one tcgen05.ld, release them, then apply bias / Q-scale / GELU / ReLU in FP32
+//     (packed FP32x2 arithmetic) and store through swizzled staging + TMA stores.  (With two groups
+//     of quads the epilogue arithmetic paced the whole kernel.)
+//   * warp 24 issues every load and owns the TMEM allocation.
 // Grid: x = piece (a tile-row range of one segment), y = 128-token block, z = K part (split-K,
 // fp32 partial outputs, reduced by the LayerNorm kernel).
 #include <cuda.h>
@@ -38,10 +39,9 @@ namespace et {
 
 #ifdef ET_TIMELINE
 // Debug builds only: %clock64 stamps (SM cycles) of CTA (0, 0, 0) of the most recent launch.
-//   slot 0: start; 1: metadata staged; 2..13: A chunk j copied to TMEM (producer); 14: last tile chunk
-//   issued; 16 + 24*w + 3*k + {0,1,2}: MMA warp w, round k: accumulator free / first MMA / commit;
-//   208 + 40*g + 5*k + {0,1,2,3}: epilogue group g, round k: quad complete / drained / math done /
-//   stores issued; 300: end.
+//   slot 0: start; 1: metadata staged; 14: last load issued; 16 + 24*w + 3*k + {0,1,2}: MMA warp w,
+//   round k: accumulator free / first MMA / commit; 208 + 40*g + 5*k + {0,1,2,3}: epilogue group g,
+//   round k: pair complete / drained / math done / stores issued; 500: end.
 __device__ unsigned long long g_timeline[512];
 __device__ __forceinline__ unsigned long long gtime() {
   unsigned long long t;
@@ -59,25 +59,26 @@ __device__ __forceinline__ unsigned long long gtime() {
 namespace {
 
 constexpr int kMaxPieces = 64;
-#ifndef ET_GEMM_NXS
-#define ET_GEMM_NXS 3
+#ifndef ET_GEMM_SLOTS
+#define ET_GEMM_SLOTS 9
 #endif
-#ifndef ET_GEMM_NBS
-#define ET_GEMM_NBS 8
-#endif
-constexpr int kNXS = ET_GEMM_NXS;   // X staging stages (16 KB each: 128 rows x 64 K)
-constexpr int kNBS = ET_GEMM_NBS;   // tile staging stages
-constexpr int kChunkTiles = 32;  // tiles per stage (16 KB)
+// Unified staging ring: the A chunks of the K part (128 rows x 64 K, SWIZZLE_128B) come first in the
+// load sequence, then the tile chunks (32 packed tiles each).  Every A load is in flight at once during
+// the prologue (the whole ring is free then), and the slots are reused for tiles as soon as the
+// fill warps have moved their A chunk into TMEM.
+constexpr int kSlots = ET_GEMM_SLOTS;
+constexpr int kSlotBytes = 16384;
+constexpr int kChunkTiles = 32;  // tiles per tile chunk (16 KB)
 constexpr int kMaxKChunks = 12;  // K <= 768 per part
 constexpr int kMaxBChunks = 192; // tile chunks per CTA (one single-use full barrier each)
 constexpr int kMaxRows = 256;    // tile rows per CTA (row pointers and bias staged in smem)
 constexpr int kAccCol = 384;     // first accumulator column (A uses [0, Kp/2) <= 384)
 constexpr int kMmaWarps = 8;     // warps 0-7: MMA issue, one accumulator (16 TMEM columns) each
-// warps 8-15: epilogue, two groups of 4 (one per TMEM lane quarter)
-constexpr int kWarpA = 16;       // A producer: TMA of the X block into the smem ring
-constexpr int kWarpB = 17;       // tile producer + TMEM owner
-constexpr int kWarpCp = 18;      // A producer: tcgen05.cp smem -> TMEM (runs behind the TMA thread)
-constexpr int kThreads = 19 * 32;
+constexpr int kEpiGroups = 4;    // warps 8-23: epilogue, 4 groups of 4 (one warp per TMEM lane quarter);
+constexpr int kEpiWarps = 16;    //   group g drains the accumulators of MMA warps 2g and 2g + 1
+constexpr int kWarpP = kMmaWarps + kEpiWarps;   // warp 24: loads (A by TMA, tiles by bulk copy), TMEM owner
+constexpr int kFillSets = kWarpP / 4;           // warps 0-23 in 6 sets of 4 move A chunks smem -> TMEM
+constexpr int kThreads = (kWarpP + 1) * 32;
 
 struct SegDev {
   const int32_t* prp;       // part_row_ptr [kparts][tile_rows + 1]
@@ -108,22 +109,24 @@ struct Params {
 };
 
 struct __align__(8) Barriers {
-  // xfull: one single-use barrier per A chunk (a fill warp may run several ring laps ahead, and a
+  // single-use barriers per A chunk / tile chunk (a warp may run laps ahead of a slot's reuse, and a
   // parity wait on a reused barrier cannot tell those phases apart)
-  uint64_t xfull[kMaxKChunks], xempty[kNXS], afill[kMaxKChunks];
+  uint64_t xfull[kMaxKChunks];   // A chunk j landed in its slot (TMA transaction bytes)
+  uint64_t xfree[kMaxKChunks];   // A chunk j read out of its slot (4 fill warps)
+  uint64_t afill[kMaxKChunks];   // A chunk j stored into TMEM (4 fill warps)
   uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
   uint64_t bfull[kMaxBChunks];
-  alignas(16) int tcol[kNBS][kChunkTiles + 4];   // (bulk-copy destination: 16-byte aligned) tile columns of the staged tiles (from a 16-byte aligned start)
+  alignas(16) int tcol[kSlots][kChunkTiles + 4];   // bulk-copy destination (16-byte aligned): tile columns
   int rptr[kMaxRows + 1];        // this CTA's row pointers, relative to its first tile
   uint32_t bias_s[kMaxRows * 8]; // this CTA's bias slice (16-bit pairs)
   uint32_t tmem_base;
-  int rows_seen[2];   // per epilogue group: rows whose MMAs were observed complete (in row order)
+  int rows_seen[kEpiGroups];     // per epilogue group: rows whose MMAs were observed complete (in order)
 };
 
-constexpr size_t kSmemX = (size_t)kNXS * 16384;
-constexpr size_t kSmemB = (size_t)kNBS * kChunkTiles * 512;
-constexpr size_t kSmemStage = 8 * 4096;   // epilogue staging: 32 rows x 128 B per epilogue warp (SW128)
-constexpr size_t kSmemBytes = 1024 + kSmemX + kSmemB + kSmemStage + sizeof(Barriers);
+constexpr size_t kSmemRing = (size_t)kSlots * kSlotBytes;
+constexpr size_t kSmemStage = (size_t)kEpiWarps * 4096;   // 32 rows x 128 B per epilogue warp
+constexpr size_t kSmemBytes = 1024 + kSmemRing + kSmemStage + sizeof(Barriers);
+static_assert(kSmemBytes <= 232448, "shared memory budget");
 
 // GELU(x) = x Phi(x) = 0.5 x (1 + erf(x / sqrt 2)) (reading C-12), evaluated as
 //   GELU(x) = max(x, 0) - |x| e,   e = 0.5 erfc(t) = 2^(-g(t) - 1),   t = |x| / sqrt 2 (clamped to 4)
@@ -156,10 +159,9 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   // 1024-byte aligned, derived from smem_raw by pointer arithmetic so the compiler keeps the shared
   // address space (an integer round trip would turn every access into a generic LD/ST)
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint8_t* sX = smem;
-  uint8_t* sB = smem + kSmemX;
-  uint8_t* sStage = smem + kSmemX + kSmemB;
-  Barriers& bar = *reinterpret_cast<Barriers*>(smem + kSmemX + kSmemB + kSmemStage);
+  uint8_t* ring = smem;
+  uint8_t* sStage = smem + kSmemRing;
+  Barriers& bar = *reinterpret_cast<Barriers*>(smem + kSmemRing + kSmemStage);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -177,30 +179,20 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
   if (threadIdx.x == 0) ET_TL(0);
   if (threadIdx.x == 0) {
-#ifndef ET_GEMM_CP_FILL
-    constexpr int kFillArrivals = 4;   // four register-fill warps per chunk
-#else
-    constexpr int kFillArrivals = 1;   // one tcgen05.commit per chunk
-#endif
-    for (int i = 0; i < kNXS; ++i) mbar_init(&bar.xempty[i], kFillArrivals);
-    for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.xfull[i], 1);
-#ifndef ET_GEMM_CP_FILL
-    for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.afill[i], kFillArrivals);
-#else
-    for (int i = 0; i < kMaxKChunks; ++i) mbar_init(&bar.afill[i], 1);
-#endif
+    for (int i = 0; i < kMaxKChunks; ++i) {
+      mbar_init(&bar.xfull[i], 1);
+      mbar_init(&bar.xfree[i], 4);
+      mbar_init(&bar.afill[i], 4);
+    }
     for (int i = 0; i < kMmaWarps; ++i) {
       mbar_init(&bar.acc_full[i], 1);
       mbar_init(&bar.acc_empty[i], 4);
     }
-    // one full barrier per tile chunk, each completing exactly once (parity 0): a warp may skip
-    // ahead to a chunk whose ring slot has not even received its previous fill, and a parity wait
-    // on a reused barrier cannot tell those phases apart.
     for (int i = 0; i < nchunks; ++i) mbar_init(&bar.bfull[i], 1);
-    bar.rows_seen[0] = bar.rows_seen[1] = 0;
+    for (int g = 0; g < kEpiGroups; ++g) bar.rows_seen[g] = 0;
     fence_mbar_init();
   }
-  if (warp == kWarpB) tmem_alloc<512>(&bar.tmem_base);
+  if (warp == kWarpP) tmem_alloc<512>(&bar.tmem_base);
   // stage the per-CTA metadata once (one global round trip instead of one per tile row)
   for (int i = threadIdx.x; i <= nrows; i += blockDim.x) bar.rptr[i] = rp[pc.i0 + i] - pb;
   if constexpr (kEpi != ET_EPI_F32) {
@@ -214,20 +206,18 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const uint32_t tbase = bar.tmem_base;
   if (threadIdx.x == 0) ET_TL(1);
 
-#ifndef ET_GEMM_CP_FILL
-  if (warp < 16) {
-    // smem ring -> TMEM through registers (instead of tcgen05.cp): chunk j is moved by the four
-    // warps with w / 4 == j % 4, warp w taking TMEM lane quarter w % 4 (its 32 token rows); lane i
-    // reads its row's 128 bytes from the SWIZZLE_128B chunk (16-byte unit c of row r sits at unit
-    // c ^ (r % 8): conflict-free) and one tcgen05.st.32x32b.x32 writes 32 packed columns.
+  if (warp < kWarpP) {
+    // A fill, smem ring -> TMEM through registers: chunk j is moved by the four warps of set j % 6,
+    // warp w taking TMEM lane quarter w % 4 (its 32 token rows); lane i reads its row's 128 bytes from
+    // the SWIZZLE_128B chunk (16-byte unit c of row r sits at unit c ^ (r % 8): conflict-free) and
+    // one tcgen05.st.32x32b.x32 writes 32 packed columns.
     const int q = warp & 3;
     const int rr = q * 32 + lane;
     const uint32_t tq = tbase + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
-    for (int j = warp >> 2; j < nk; j += 4) {
-      const int slot = j % kNXS;
+    for (int j = warp >> 2; j < nk; j += kFillSets) {
       mbar_wait_warp(&bar.xfull[j], 0);
-      const uint8_t* rowp = sX + slot * 16384 + rr * 128;
+      const uint8_t* rowp = ring + (j % kSlots) * kSlotBytes + rr * 128;
       uint32_t v[32];
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
@@ -235,7 +225,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         v[4 * c] = u.x; v[4 * c + 1] = u.y; v[4 * c + 2] = u.z; v[4 * c + 3] = u.w;
       }
       __syncwarp();
-      if (lane == 0) mbar_arrive(&bar.xempty[slot]);   // the TMA thread may refill the slot
+      if (lane == 0) mbar_arrive(&bar.xfree[j]);   // the producer may reuse the slot
       tmem_st32(tq + j * 32, v);
       tmem_st_wait();
       tc_fence_before();
@@ -243,76 +233,51 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       if (lane == 0) mbar_arrive(&bar.afill[j]);
     }
   }
-  if (warp == kWarpCp) {
-    // idle in this build
-  } else
-#endif
-  if (warp == kWarpA) {
-    // ===================== A producer (TMA): X block -> smem ring, up to kNXS chunks ahead
+
+  if (warp == kWarpP) {
+    // ===================== producer: A chunks (TMA) then tile chunks (bulk copies) through the ring.
+    // Slot reuse: an A slot once its chunk was read out; a tile slot once every tile row touching
+    // the old chunk completed its MMAs (row-granular; epilogue group g publishes rows_seen[g], its
+    // rows being 8k + 2g + {0, 1}).  A row spans at most 3 tile chunks < kSlots, so the producer
+    // never waits for a row that itself needs the chunk being loaded.
     if (lane == 0) {
       tma_prefetch_desc(&tmap_x);
       const int kx0 = z * p.Kp;
-      for (int j = 0; j < nk; ++j) {
-        const int slot = j % kNXS;
-        if (j >= kNXS) mbar_wait(&bar.xempty[slot], ((j / kNXS) - 1) & 1);
-        mbar_expect_tx(&bar.xfull[j], p.box_rows * 128);
-        tma_load_2d(sX + slot * 16384, &tmap_x, &bar.xfull[j], kx0 + j * 64, m0);
-      }
-    }
-  } else if (warp == kWarpCp) {
-    // ===================== A producer (copy): smem ring -> TMEM columns [32 j, 32 j + 32)
-    if (lane == 0) {
-      for (int j = 0; j < nk; ++j) {
-        const int slot = j % kNXS;
-        mbar_wait(&bar.xfull[j], 0);
-        tc_fence_after();
-        const uint32_t src = smem_u32(sX + slot * 16384);
-#pragma unroll
-        for (int s = 0; s < 4; ++s)
-          tmem_cp_128x256b(tbase + j * 32 + s * 8, make_sdesc(src + s * 32, 16, 1024, kLayoutSW128));
-        mma_commit(&bar.afill[j]);       // chunk j readable by the MMA warps
-        mma_commit(&bar.xempty[slot]);   // smem slot free for the TMA thread
-#ifdef ET_TIMELINE
-        mbar_wait(&bar.afill[j], 0);
-        ET_TL(2 + j);
-#endif
-      }
-    }
-  } else if (warp == kWarpB) {
-    // ===================== tile producer: packed tiles -> smem ring (bulk copies)
-    // Slot reuse is row-granular: chunk c may overwrite chunk c - kNBS once every tile row touching
-    // chunk c - kNBS has completed its MMAs.  Epilogue group g owns rows 8k + 4g + a (a < 4) and
-    // publishes rows_seen[g] in that order.  (A single row spans at most 3 chunks < kNBS, so the
-    // producer never waits for a row that itself needs the chunk being loaded.)
-    if (lane == 0) {
       const uint8_t* vals = sg.values + (size_t)pb * 512;
-      int tl = 0;   // last local row that starts before the end of the chunk being recycled
-      // Chunks beyond what round 0 needs wait until the A block is in TMEM: in the prologue every
-      // CTA of the grid streams its A block at once and the chip's L2 bandwidth is the limit, so
-      // tile prefetch would only delay the first MMAs.
-      const int c_r0 = (bar.rptr[min(kMmaWarps, nrows)] + kChunkTiles - 1) / kChunkTiles + 1;
-      for (int c = 0; c < nchunks; ++c) {
-        const int slot = c % kNBS;
-#ifndef ET_GEMM_EAGER_B
-        if (c == c_r0) mbar_wait(&bar.afill[nk - 1], 0);
-#endif
-        if (c >= kNBS) {
-          const int end_tile = pb + (c - kNBS + 1) * kChunkTiles;
-          while (tl + 1 < nrows && bar.rptr[tl + 1] + pb < end_tile) ++tl;
-          const int full = (tl + 1) / kMmaWarps, rem = (tl + 1) % kMmaWarps;
-          const int need0 = 4 * full + min(max(rem, 0), 4);
-          const int need1 = 4 * full + min(max(rem - 4, 0), 4);
-          while (ld_acquire_shared(&bar.rows_seen[0]) < need0) {}
-          while (ld_acquire_shared(&bar.rows_seen[1]) < need1) {}
+      int tl = 0;   // last local row that starts before the end of the tile chunk being recycled
+      const int nseq = nk + nchunks;
+      for (int s = 0; s < nseq; ++s) {
+        const int slot = s % kSlots;
+        const int prev = s - kSlots;
+        if (prev >= 0) {
+          if (prev < nk) {
+            mbar_wait(&bar.xfree[prev], 0);
+          } else {
+            const int end_rel = (prev - nk + 1) * kChunkTiles;
+            while (tl + 1 < nrows && bar.rptr[tl + 1] < end_rel) ++tl;
+            const int full = (tl + 1) / kMmaWarps, rem = (tl + 1) % kMmaWarps;
+#pragma unroll
+            for (int g = 0; g < kEpiGroups; ++g) {
+              const int need = 2 * full + min(max(rem - 2 * g, 0), 2);
+              while (ld_acquire_shared(&bar.rows_seen[g]) < need) {}
+            }
+          }
         }
-        const int nt = min(kChunkTiles, pe - pb - c * kChunkTiles);
-        // tile columns: copy from the 16-byte aligned start at or below the chunk's first entry
-        // (tile_col is allocated with 16 bytes of slack, et_prune_pack_query)
-        const int first = pb + c * kChunkTiles, off = first & 3;
-        const int col_bytes = ((off + nt) * 4 + 15) & ~15;
-        mbar_expect_tx(&bar.bfull[c], nt * 512 + col_bytes);
-        bulk_load(sB + slot * (kChunkTiles * 512), vals + (size_t)c * kChunkTiles * 512, nt * 512, &bar.bfull[c]);
-        bulk_load(&bar.tcol[slot][0], sg.tile_col + (first - off), col_bytes, &bar.bfull[c]);
+        uint8_t* dst = ring + slot * kSlotBytes;
+        if (s < nk) {
+          mbar_expect_tx(&bar.xfull[s], p.box_rows * 128);
+          tma_load_2d(dst, &tmap_x, &bar.xfull[s], kx0 + s * 64, m0);
+        } else {
+          const int c = s - nk;
+          const int nt = min(kChunkTiles, pe - pb - c * kChunkTiles);
+          // tile columns: copy from the 16-byte aligned start at or below the chunk's first entry
+          // (tile_col is allocated with 16 bytes of slack, et_prune_pack_query)
+          const int first = pb + c * kChunkTiles, off = first & 3;
+          const int col_bytes = ((off + nt) * 4 + 15) & ~15;
+          mbar_expect_tx(&bar.bfull[c], nt * 512 + col_bytes);
+          bulk_load(dst, vals + (size_t)c * kChunkTiles * 512, nt * 512, &bar.bfull[c]);
+          bulk_load(&bar.tcol[slot][0], sg.tile_col + (first - off), col_bytes, &bar.bfull[c]);
+        }
       }
       ET_TL(14);
     }
@@ -320,10 +285,10 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     // ===================== MMA warps: warp w issues the chains of tile rows w, w+8, w+16, ...
     const uint32_t idesc = make_idesc_f16(128, 16, kBF16 ? 1 : 0, 0, 0);
     const uint32_t d_tmem = tbase + kAccCol + warp * 16;
-    const uint32_t sB_u32 = smem_u32(sB);
+    const uint32_t ring_u32 = smem_u32(ring);
     const int kbase = z * 48;   // first tile column of this K part
     int a_ready = -1;           // highest A chunk known filled
-    int cur_chunk = -1;         // B chunk whose full barrier was last waited
+    int cur_chunk = -1;         // tile chunk whose full barrier was last waited
     for (int k = 0; k < nrounds; ++k) {
       const int t = k * kMmaWarps + warp;
       if (t >= nrows) break;
@@ -342,7 +307,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           cur_chunk = c;
           tc_fence_after();
         }
-        const int slot = c % kNBS;
+        const int slot = (nk + c) % kSlots;
         const int coff = (pb + c * kChunkTiles) & 3;
         n = qe - qb;
         const int mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
@@ -354,7 +319,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           tc_fence_after();
         }
         // B descriptor of tile u: start address field advances by 512 B / 16 = 32 per tile
-        const uint64_t bd0 = make_sdesc(sB_u32 + slot * (kChunkTiles * 512) + (qb % kChunkTiles) * 512, 128, 256,
+        const uint64_t bd0 = make_sdesc(ring_u32 + slot * kSlotBytes + (qb % kChunkTiles) * 512, 128, 256,
                                         kLayoutNone);
         blo = (uint32_t)bd0;
         bhi = (uint32_t)(bd0 >> 32);
@@ -386,37 +351,35 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k + 2);
     }
   } else {
-    // ===================== epilogue warps: group g drains the accumulators of MMA warps 4g..4g+3
-    const int g = (warp - kMmaWarps) >> 2;
+    // ===================== epilogue warps: group g drains the accumulators of MMA warps 2g, 2g+1
+    const int ew = warp - kMmaWarps;
+    const int g = ew >> 2;
     const int quarter = warp & 3;               // TMEM lane quarter this warp may access
-    // Per round: wait for the group's 4 accumulators (rows 8k + 4g + a), read all 64 columns with
+    uint8_t* st = sStage + ew * 4096;
+    // Per round: wait for the group's 2 accumulators (rows 8k + 2g + a), read their 32 columns with
     // one TMEM load, release them to the MMA warps, THEN do the bias / activation / store math (so
     // an MMA warp never waits for another row's epilogue arithmetic).
     for (int k = 0; k < nrounds; ++k) {
-      const int t0 = k * kMmaWarps + g * 4;   // first row of this group's quad in round k
+      const int t0 = k * kMmaWarps + g * 2;   // first row of this group's pair in round k
       if (t0 >= nrows) break;
-      const int na = min(4, nrows - t0);
-      uint32_t r[64];
-      for (int a = 0; a < na; ++a) {
-        mbar_wait_warp(&bar.acc_full[g * 4 + a], k & 1);
-      }
+      const int na = min(2, nrows - t0);
+      uint32_t r[32];
+      for (int a = 0; a < na; ++a) mbar_wait_warp(&bar.acc_full[g * 2 + a], k & 1);
       if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k);
       tc_fence_after();
       if (quarter == 0 && lane == 0)
-        st_release_shared(&bar.rows_seen[g], k * 4 + na);   // rows' MMAs complete: their B tiles are free
-      tmem_ld32(tbase + kAccCol + g * 64 + ((uint32_t)(quarter * 32) << 16), *reinterpret_cast<uint32_t(*)[32]>(r));
-      tmem_ld32(tbase + kAccCol + g * 64 + 32 + ((uint32_t)(quarter * 32) << 16),
-                *reinterpret_cast<uint32_t(*)[32]>(r + 32));
+        st_release_shared(&bar.rows_seen[g], k * 2 + na);   // rows' MMAs complete: their tiles are free
+      tmem_ld32(tbase + kAccCol + g * 32 + ((uint32_t)(quarter * 32) << 16), r);
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
       if (lane == 0)
-        for (int a = 0; a < na; ++a) mbar_arrive(&bar.acc_empty[g * 4 + a]);
+        for (int a = 0; a < na; ++a) mbar_arrive(&bar.acc_empty[g * 2 + a]);
       if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 1);
-      // math: bias / scale / activation on the quad's 64 columns of this thread's token row
-      float v[64];
+      // math: bias / scale / activation on the pair's 32 columns of this thread's token row
+      float v[32];
 #pragma unroll
-      for (int a = 0; a < 4; ++a) {
+      for (int a = 0; a < 2; ++a) {
         const int t = t0 + min(a, na - 1);
         const bool empty_row = a >= na || bar.rptr[t + 1] == bar.rptr[t];
 #pragma unroll
@@ -445,59 +408,53 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         }
       }
       if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 2);
-      // store: registers -> this warp's 32-row staging tile (128 B rows, SWIZZLE_128B, conflict-free)
-      // -> one TMA tensor store per 128-byte column block (clipped at M by the tensor map)
-      uint8_t* st = sStage + (warp - kMmaWarps) * 4096;
+      // store: registers -> this warp's 32-row staging tile -> one TMA tensor store (clipped at M by
+      // the tensor map).  fp32: 128-byte rows, SWIZZLE_128B (unit c of row r at c ^ (r % 8));
+      // 16-bit: 64-byte rows, SWIZZLE_64B (unit c of row r at c ^ ((r / 2) % 4)); both conflict-free.
       const int col0 = sg.out_col + (pc.i0 + t0) * 16;
       const int row0 = m0 + quarter * 32;
-      constexpr int kPasses = kEpi == ET_EPI_F32 ? 2 : 1;   // fp32: 32 columns (128 B) per pass
-      if (na == 4) {
+      if (na == 2) {
+        if (lane == 0) bulk_wait_group_read<0>();   // the previous store finished reading the staging tile
+        __syncwarp();
+        if constexpr (kEpi == ET_EPI_F32) {
 #pragma unroll
-        for (int ps = 0; ps < kPasses; ++ps) {
-          if (lane == 0) bulk_wait_group_read<0>();   // previous store finished reading the staging tile
-          __syncwarp();
-#pragma unroll
-          for (int ch = 0; ch < 8; ++ch) {   // 8 x 16-byte chunks of this row's 128 bytes
-            uint4 u;
-            if constexpr (kEpi == ET_EPI_F32) {
-              const float* f = v + ps * 32 + ch * 4;
-              u = make_uint4(__float_as_uint(f[0]), __float_as_uint(f[1]), __float_as_uint(f[2]),
-                             __float_as_uint(f[3]));
-            } else {
-              const float* f = v + ch * 8;
-              u = make_uint4(pack2<kBF16>(f[0], f[1]), pack2<kBF16>(f[2], f[3]), pack2<kBF16>(f[4], f[5]),
-                             pack2<kBF16>(f[6], f[7]));
-            }
-            *reinterpret_cast<uint4*>(st + lane * 128 + ((ch ^ (lane & 7)) << 4)) = u;
+          for (int ch = 0; ch < 8; ++ch) {
+            const float* f = v + ch * 4;
+            *reinterpret_cast<uint4*>(st + lane * 128 + ((ch ^ (lane & 7)) << 4)) =
+                make_uint4(__float_as_uint(f[0]), __float_as_uint(f[1]), __float_as_uint(f[2]), __float_as_uint(f[3]));
           }
-          fence_proxy_async_smem();
-          __syncwarp();
-          if (lane == 0) {
-            if constexpr (kEpi == ET_EPI_F32) tma_store_3d(&tmap_y, st, col0 + ps * 32, row0, z);
-            else tma_store_2d(&tmap_y, st, col0, row0);
-            bulk_commit_group();
+        } else {
+#pragma unroll
+          for (int ch = 0; ch < 4; ++ch) {
+            const float* f = v + ch * 8;
+            *reinterpret_cast<uint4*>(st + lane * 64 + ((ch ^ ((lane >> 1) & 3)) << 4)) =
+                make_uint4(pack2<kBF16>(f[0], f[1]), pack2<kBF16>(f[2], f[3]), pack2<kBF16>(f[4], f[5]),
+                           pack2<kBF16>(f[6], f[7]));
           }
         }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          if constexpr (kEpi == ET_EPI_F32) tma_store_3d(&tmap_y, st, col0, row0, z);
+          else tma_store_2d(&tmap_y, st, col0, row0);
+          bulk_commit_group();
+        }
       } else {
-        // partial quad (last rows of a segment): direct stores of the valid 16-column groups only,
-        // so nothing is written into the neighbouring segment's columns
+        // a lone last row of the piece: direct stores of its 16 columns only, so nothing is written
+        // into the neighbouring piece's or segment's columns
         const int row = row0 + lane;
         if (row < p.M) {
-          for (int a = 0; a < na; ++a) {
-            if constexpr (kEpi == ET_EPI_F32) {
-              float* y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row * p.ldy + col0 + a * 16;
+          if constexpr (kEpi == ET_EPI_F32) {
+            float* y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row * p.ldy + col0;
 #pragma unroll
-              for (int c = 0; c < 16; c += 4)
-                *reinterpret_cast<float4*>(y + c) = make_float4(v[a * 16 + c], v[a * 16 + c + 1], v[a * 16 + c + 2],
-                                                               v[a * 16 + c + 3]);
-            } else {
-              uint16_t* y = static_cast<uint16_t*>(p.Y) + (size_t)row * p.ldy + col0 + a * 16;
-              const float* f = v + a * 16;
-              *reinterpret_cast<uint4*>(y) = make_uint4(pack2<kBF16>(f[0], f[1]), pack2<kBF16>(f[2], f[3]),
-                                                        pack2<kBF16>(f[4], f[5]), pack2<kBF16>(f[6], f[7]));
-              *reinterpret_cast<uint4*>(y + 8) = make_uint4(pack2<kBF16>(f[8], f[9]), pack2<kBF16>(f[10], f[11]),
-                                                            pack2<kBF16>(f[12], f[13]), pack2<kBF16>(f[14], f[15]));
-            }
+            for (int c = 0; c < 16; c += 4)
+              *reinterpret_cast<float4*>(y + c) = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+          } else {
+            uint16_t* y = static_cast<uint16_t*>(p.Y) + (size_t)row * p.ldy + col0;
+            *reinterpret_cast<uint4*>(y) = make_uint4(pack2<kBF16>(v[0], v[1]), pack2<kBF16>(v[2], v[3]),
+                                                      pack2<kBF16>(v[4], v[5]), pack2<kBF16>(v[6], v[7]));
+            *reinterpret_cast<uint4*>(y + 8) = make_uint4(pack2<kBF16>(v[8], v[9]), pack2<kBF16>(v[10], v[11]),
+                                                          pack2<kBF16>(v[12], v[13]), pack2<kBF16>(v[14], v[15]));
           }
         }
       }
@@ -505,12 +462,12 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     }
   }
 
-  if (warp >= kMmaWarps && warp < kMmaWarps + 8 && lane == 0) bulk_wait_group<0>();   // epilogue stores done
-  __syncwarp();   // producer warps: lane 0 ran the loops alone; reconverge before the block barrier
+  if (warp >= kMmaWarps && warp < kWarpP && lane == 0) bulk_wait_group<0>();   // epilogue stores done
+  __syncwarp();   // the producer warp: lane 0 ran the loop alone; reconverge before the block barrier
   tc_fence_before();
   __syncthreads();
-  if (threadIdx.x == 0) ET_TL(300);
-  if (warp == kWarpB) {
+  if (threadIdx.x == 0) ET_TL(500);
+  if (warp == kWarpP) {
     __syncwarp();
     tc_fence_after();
     tmem_dealloc<512>(tbase);   // .sync.aligned: the whole warp, converged
@@ -674,15 +631,15 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   CUtensorMap tm;   // the K offset k0 is folded into the base address
   ET_TRY(make_tmap_2d(&tm, static_cast<const uint8_t*>(a.X) + (size_t)a.k0 * 2, a.dtype, (uint64_t)a.M,
                       (uint64_t)a.K, (uint64_t)a.ldx, 64, (uint32_t)prm.box_rows, true));
-  // output tensor map: [M, ldy] in the operand dtype, box 64 cols x 32 rows (one epilogue warp's
-  // staging tile); fp32 partials: [kparts, M, ldy], box 32 x 32 x 1.  SWIZZLE_128B staging.
+  // output tensor map: [M, ldy] in the operand dtype, box 32 cols x 32 rows (one epilogue warp's
+  // staging tile, SWIZZLE_64B); fp32 partials: [kparts, M, ldy], box 32 x 32 x 1 (SWIZZLE_128B).
   CUtensorMap tmy;
   if (a.epi == ET_EPI_F32) {
     ET_TRY(make_tmap_3d_f32(&tmy, a.Y, (uint64_t)a.ldy, (uint64_t)a.M, (uint64_t)kparts, 32,
                             a.M < 32 ? (uint32_t)a.M : 32u));
   } else {
-    ET_TRY(make_tmap_2d(&tmy, a.Y, a.dtype, (uint64_t)a.M, (uint64_t)a.ldy, (uint64_t)a.ldy, 64,
-                        a.M < 32 ? (uint32_t)a.M : 32u, true));
+    ET_TRY(make_tmap_2d_sw64(&tmy, a.Y, a.dtype, (uint64_t)a.M, (uint64_t)a.ldy, (uint64_t)a.ldy, 32,
+                             a.M < 32 ? (uint32_t)a.M : 32u));
   }
   dim3 grid(np, mblocks, kparts);
   const bool bf = a.dtype == ET_BF16;

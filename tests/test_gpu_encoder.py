@@ -134,3 +134,27 @@ def test_invalid_arguments_fail_loudly(etm):
         etm.attn_core_fwd(qkv, 1, 512, 12, 768, 0, 768, 1536, mode="short")   # short form needs S <= 256
     with pytest.raises(etm.EtError):
         etm.Encoder([layer], 1, 128, 12, cfg.d_ff, resid_dtype="bf16")  # resid must be fp32 or fp16 here
+
+
+@pytest.mark.parametrize("key,kw", [("C3", {"layers": 2, "batch": 4}), ("C4", {"layers": 1, "batch": 2})])
+def test_graph_replay_bitexact(etm, key, kw):
+    """et_encoder_graph_create / et_graph_launch replays exactly the kernels of et_encoder_fwd:
+    bit-identical output, and X is re-read at every launch (refilled in place)."""
+    cfg, raws, X, lens = _case(key, **kw)
+    Y0, enc, Xd = _gpu(etm, cfg, raws, X, lens)
+    out = torch.empty_like(Xd)
+    g = enc.capture(Xd, out)
+    n0 = etm._lib.et_launch_count()
+    enc(Xd, torch.empty_like(Xd))
+    n_direct = etm._lib.et_launch_count() - n0
+    n0 = etm._lib.et_launch_count()
+    g.launch()
+    torch.cuda.synchronize()
+    assert etm._lib.et_launch_count() - n0 == n_direct >= 7 * cfg.layers
+    assert np.array_equal(to64(out).reshape(Y0.shape), Y0)
+    X2 = make_x(cfg, seed=1234)
+    Xd.copy_(dev_tensor(X2.reshape(cfg.tokens, cfg.d_model), cfg.dtype))
+    g.launch()
+    Y2 = enc(Xd.clone())
+    torch.cuda.synchronize()
+    assert np.array_equal(to64(out), to64(Y2))
