@@ -324,8 +324,9 @@ def our_arm(args):
     graph = enc.capture(Xd, out)
     K = args.steps
     cap = len(layers) * 8 + 4
-    et._check(et._lib.et_trace_begin(cap))
-    graph_tr = enc.capture(Xd, out)       # same kernels + external event-record nodes per kernel
+    slots = torch.empty(2 * cap, dtype=torch.int64, device="cuda")   # device-side kernel spans (et.h tracing)
+    et._check(et._lib.et_trace_begin(cap, slots.data_ptr()))
+    graph_tr = enc.capture(Xd, out)       # same kernels, each stamping its device span into `slots`
     n_int = __import__("ctypes").c_int32()
     et._check(et._lib.et_trace_end(__import__("ctypes").byref(n_int)))
     for _ in range(max(args.warmup, 3)):
@@ -352,6 +353,7 @@ def our_arm(args):
     t_local = sum(step_ms) / 1e3
 
     # ---------------- per-kernel device time: K replays of the traced graph, same flush discipline
+    # (every kernel's span = first CTA start to last CTA end, from %globaltimer inside the kernels)
     import ctypes
     kind = ctypes.c_int32()
     ms = ctypes.c_float()
@@ -359,6 +361,7 @@ def our_arm(args):
     tr_ms = []
     for s in range(K):
         flush.fill_(float(s))
+        slots.fill_(-1)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         graph_tr.launch()

@@ -242,20 +242,24 @@ et_status et_graph_launch(et_graph* graph, void* stream);
 et_status et_graph_destroy(et_graph* graph);
 
 /* ------------------------------------------------------------------------------------------
- * Tracing (calling thread only): while enabled, the forward entry points record a CUDA event on
- * the caller's stream before every kernel they launch (and one after the last), tagged with the
- * step kind, so that per-kernel device time can be read back after the stream is synchronised.
- * Event handles are created lazily by the library (no device memory).  Recording stops silently
- * once `capacity` marks have been taken.
+ * Tracing (calling thread only; diagnostics, not part of the metric): while enabled, every kernel
+ * the forward entry points launch (or capture into a graph) is given one slot of two uint64 in
+ * `dev_slots` (caller-allocated device memory, 2 * capacity entries).  Thread 0 of each CTA of
+ * that kernel folds %globaltimer (ns) into slot[0] with atomicMin when it starts and
+ * ~%globaltimer into slot[1] with atomicMin when it ends, so the caller must fill the slots with
+ * all-one bytes (e.g. cudaMemsetAsync(dev_slots, 0xFF, ...)) before every traced run.  The slot
+ * then holds the kernel's device span: first CTA start to last CTA end.  Launches beyond
+ * `capacity` are not traced.
  * ------------------------------------------------------------------------------------------ */
 typedef enum {
   ET_K_QKV = 0, ET_K_ATTN = 1, ET_K_OPROJ = 2, ET_K_LN1 = 3, ET_K_FFN1 = 4, ET_K_FFN2 = 5, ET_K_LN2 = 6,
-  ET_K_AUX = 7, ET_K_END = 8
+  ET_K_AUX = 7
 } et_kernel_kind;
-et_status et_trace_begin(int32_t capacity);
-/* Stop recording; *n_intervals = number of recorded kernel intervals. */
-et_status et_trace_end(int32_t* n_intervals);
-/* Interval i (after synchronising the stream): its kind and device milliseconds. */
+et_status et_trace_begin(int32_t capacity, unsigned long long* dev_slots);
+/* Stop assigning slots; *n_launches = number of traced launches. */
+et_status et_trace_end(int32_t* n_launches);
+/* Traced launch i (after synchronising the stream): its kind and device milliseconds (reads the
+ * slot with a synchronous cudaMemcpy).  ET_ERR_INVALID_ARG if i is out of range or unwritten. */
 et_status et_trace_get(int32_t i, int32_t* kind, float* ms);
 /* Number of library kernels launched by this thread since process start (launch accounting). */
 int64_t et_launch_count(void);

@@ -402,7 +402,7 @@ def encoder_fwd(X: torch.Tensor, layers: list, batch: int, seq_len: int, heads: 
 
 
 # ------------------------------------------------------------------------------------------ tracing
-_sig("et_trace_begin", ctypes.c_int, [_i32])
+_sig("et_trace_begin", ctypes.c_int, [_i32, _vp])
 _sig("et_trace_end", ctypes.c_int, [ctypes.POINTER(_i32)])
 _sig("et_trace_get", ctypes.c_int, [_i32, ctypes.POINTER(_i32), ctypes.POINTER(_f32)])
 _sig("et_launch_count", ctypes.c_int64, [])

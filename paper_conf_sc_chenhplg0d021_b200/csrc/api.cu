@@ -33,10 +33,13 @@ et_status fail(et_status s, const char* fmt, ...) {
 }
 
 // ---------------------------------------------------------------- tracing
+// Device-side trace: every traced launch gets a slot of two u64 in caller memory; thread 0 of each
+// CTA folds %globaltimer into slot[0] with atomicMin at its start and ~%globaltimer into slot[1]
+// with atomicMin at its end (both start from all-ones), so slot = (first CTA start, last CTA end).
 struct Trace {
   bool on = false;
   int capacity = 0, n = 0;
-  std::vector<cudaEvent_t> ev;
+  unsigned long long* slots = nullptr;
   std::vector<int> kind;
 };
 static thread_local Trace g_trace;
@@ -46,23 +49,11 @@ void count_launch() { ++g_launches; }
 void add_launches(long long n) { g_launches += n; }
 long long launch_count() { return g_launches; }
 
-void trace_mark(int kind, cudaStream_t stream) {
+unsigned long long* trace_slot(int kind) {
   Trace& t = g_trace;
-  if (!t.on || t.n >= t.capacity) return;
-  if ((int)t.ev.size() <= t.n) {
-    cudaEvent_t e;
-    if (cudaEventCreate(&e) != cudaSuccess) return;
-    t.ev.push_back(e);
-    t.kind.push_back(0);
-  }
-  // inside a stream capture the event must be an external record node so that every replay of
-  // the graph records it again (a plain record would only order the capture)
-  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-  cudaStreamIsCapturing(stream, &cs);
-  if (cs == cudaStreamCaptureStatusActive) cudaEventRecordWithFlags(t.ev[t.n], stream, cudaEventRecordExternal);
-  else cudaEventRecord(t.ev[t.n], stream);
+  if (!t.on || t.n >= t.capacity) return nullptr;
   t.kind[t.n] = kind;
-  ++t.n;
+  return t.slots + 2 * (size_t)t.n++;
 }
 
 static bool valid_dtype(et_dtype d) { return d == ET_FP16 || d == ET_BF16 || d == ET_FP32; }
@@ -84,26 +75,32 @@ extern "C" {
 const char* et_last_error(void) { return g_err.c_str(); }
 const char* et_version(void) { return "et-b200 0.1 (sm_100a)"; }
 
-et_status et_trace_begin(int32_t capacity) {
-  if (capacity < 2) return fail(ET_ERR_INVALID_ARG, "et_trace_begin: capacity < 2");
+et_status et_trace_begin(int32_t capacity, unsigned long long* dev_slots) {
+  if (capacity < 1 || !dev_slots) return fail(ET_ERR_INVALID_ARG, "et_trace_begin: capacity < 1 or null slots");
   g_trace.on = true;
   g_trace.capacity = capacity;
   g_trace.n = 0;
+  g_trace.slots = dev_slots;
+  g_trace.kind.assign(capacity, 0);
   return ET_OK;
 }
 
-et_status et_trace_end(int32_t* n_intervals) {
+et_status et_trace_end(int32_t* n_launches) {
   g_trace.on = false;
-  if (n_intervals) *n_intervals = g_trace.n > 0 ? g_trace.n - 1 : 0;
+  if (n_launches) *n_launches = g_trace.n;
   return ET_OK;
 }
 
 et_status et_trace_get(int32_t i, int32_t* kind, float* ms) {
-  if (i < 0 || i + 1 >= g_trace.n) return fail(ET_ERR_INVALID_ARG, "et_trace_get: index out of range");
+  if (i < 0 || i >= g_trace.n || !g_trace.slots) return fail(ET_ERR_INVALID_ARG, "et_trace_get: index out of range");
   if (kind) *kind = g_trace.kind[i];
   if (ms) {
-    cudaError_t e = cudaEventElapsedTime(ms, g_trace.ev[i], g_trace.ev[i + 1]);
+    unsigned long long s[2];
+    cudaError_t e = cudaMemcpy(s, g_trace.slots + 2 * (size_t)i, sizeof(s), cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) return fail(ET_ERR_CUDA, "et_trace_get: %s", cudaGetErrorString(e));
+    const unsigned long long t0 = s[0], t1 = ~s[1];
+    if (s[0] == ~0ull || s[1] == ~0ull || t1 < t0) return fail(ET_ERR_INVALID_ARG, "et_trace_get: slot %d not written", i);
+    *ms = (float)((double)(t1 - t0) * 1e-6);
   }
   return ET_OK;
 }

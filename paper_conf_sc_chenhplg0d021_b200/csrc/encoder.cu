@@ -116,7 +116,6 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   const void* bv_use = bv;
   *bo_eff = bo;
   if (rowv) {
-    trace_mark(ET_K_AUX, st);
     VPrep vp{wv, wo, bv, bo, H, dk, d->dtype, ws.v_col, ws.v_width, ws.bv_packed, ws.bo_folded};
     ET_TRY(vprep_run(vp, st));
     bv_use = ws.bv_packed;
@@ -140,7 +139,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   g.Y = ws.qkv;
   g.ldy = ws.ldq;
   g.epi = ET_EPI_BIAS_SCALE;
-  trace_mark(ET_K_QKV, st);
+  g.ts = trace_slot(ET_K_QKV);
   ET_TRY(gemm_run(g, st));
   // 2. attention core
   AttnArgs a{};
@@ -166,7 +165,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   a.v_width_max = dk;
   a.scale = 1.0f;
   a.dtype = d->dtype;
-  trace_mark(ET_K_ATTN, st);
+  a.ts = trace_slot(ET_K_ATTN);
   ET_TRY(attention_run(a, st));
   // 3. output projection -> fp32 (bias and residual are added by the LayerNorm step)
   GemmArgs o{};
@@ -180,7 +179,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   o.Y = ws.part;
   o.ldy = dm;
   o.epi = ET_EPI_F32;
-  trace_mark(ET_K_OPROJ, st);
+  o.ts = trace_slot(ET_K_OPROJ);
   return gemm_run(o, st);
 }
 
@@ -258,10 +257,9 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   ET_TRY(run_attention_block(desc, X, wq, wk, wv, wo, bq, bk, bv, bo, ws, &bo_eff, st));
   const int M = desc->batch * desc->seq_len;
   LnArgs ln{ws.part, 1, M, dm, bo_eff, desc->dtype, ln_gamma ? X : nullptr, desc->dtype, ln_gamma, ln_beta, ln_eps,
-            out, nullptr};
-  trace_mark(ET_K_LN1, st);
+            out, nullptr, nullptr};
+  ln.ts = trace_slot(ET_K_LN1);
   ET_TRY(layernorm_run(ln, st));   // gamma == NULL: out = attn = part + b_O' (no residual, no LN)
-  trace_mark(ET_K_END, st);
   return ET_OK;
 }
 
@@ -337,7 +335,6 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
   const void* cur_res = X;
   const void* cur_act = X;
   if (split) {
-    trace_mark(ET_K_AUX, st);
     ET_TRY(cast_run(X, resid_dtype, xa, desc->dtype, M * dm, st));
     cur_act = xa;
   }
@@ -349,8 +346,8 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     ET_TRY(run_attention_block(desc, cur_act, &L.wq, &L.wk, &L.wv, &L.wo, L.bq, L.bk, L.bv, L.bo, ws, &bo_eff, st));
     // 4. Y1 = LN(X + attn)
     LnArgs ln1{ws.part, 1, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,
-               y1a, split ? y1r : nullptr};
-    trace_mark(ET_K_LN1, st);
+               y1a, split ? y1r : nullptr, nullptr};
+    ln1.ts = trace_slot(ET_K_LN1);
     ET_TRY(layernorm_run(ln1, st));
     // 5. U = act(Y1 W1'^T + b1)
     GemmArgs f1{};
@@ -364,7 +361,7 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     f1.Y = U;
     f1.ldy = d_ff;
     f1.epi = act == ET_ACT_GELU_ERF ? ET_EPI_BIAS_GELU : ET_EPI_BIAS_RELU;
-    trace_mark(ET_K_FFN1, st);
+    f1.ts = trace_slot(ET_K_FFN1);
     ET_TRY(gemm_run(f1, st));
     // 6. U W2'^T -> fp32 split-K partials
     GemmArgs f2{};
@@ -378,17 +375,16 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     f2.Y = ws.part;
     f2.ldy = dm;
     f2.epi = ET_EPI_F32;
-    trace_mark(ET_K_FFN2, st);
+    f2.ts = trace_slot(ET_K_FFN2);
     ET_TRY(gemm_run(f2, st));
     // 7. Y2 = LN(Y1 + F + b2)
     LnArgs ln2{ws.part, L.w2.kparts, (int)M, dm, L.b2, desc->dtype, y1r, resid_dtype, L.ln2_g, L.ln2_b, ln_eps,
-               split ? next_act : nullptr, next_res};
-    trace_mark(ET_K_LN2, st);
+               split ? next_act : nullptr, next_res, nullptr};
+    ln2.ts = trace_slot(ET_K_LN2);
     ET_TRY(layernorm_run(ln2, st));
     cur_res = next_res;
     cur_act = split ? xa : next_res;
   }
-  trace_mark(ET_K_END, st);
   return ET_OK;
 }
 

@@ -69,6 +69,7 @@ struct GemmArgs {
   void* Y;                  // output [M, ldy] (dtype) or fp32 partials [nparts][M, ldy]
   int ldy;
   et_epilogue epi;
+  unsigned long long* ts;   // trace slot or nullptr
 };
 et_status gemm_run(const GemmArgs& a, cudaStream_t stream);
 
@@ -85,6 +86,7 @@ struct LnArgs {
   float eps;
   void* out_act;
   void* out_resid;
+  unsigned long long* ts;   // trace slot or nullptr
 };
 et_status layernorm_run(const LnArgs& a, cudaStream_t stream);
 
@@ -104,6 +106,7 @@ struct AttnArgs {
   int v_width_max;          // upper bound of the per-head V width (multiple of 16)
   float scale;
   et_dtype dtype;
+  unsigned long long* ts;   // trace slot or nullptr
 };
 et_status attention_run(const AttnArgs& a, cudaStream_t stream);
 int attn_short_max(int d_k);
@@ -128,7 +131,7 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream);
 
 // ---------------------------------------------------------------- tracing (api.cu)
 // Record a mark of `kind` on `stream` if tracing is enabled; counts one kernel launch.
-void trace_mark(int kind, cudaStream_t stream);
+unsigned long long* trace_slot(int kind);   // device slot of the next traced launch, or nullptr
 void count_launch();
 void add_launches(long long n);
 long long launch_count();

@@ -71,6 +71,7 @@ struct AParams {
   float scale_log2;         // scale * log2(e)
   int box_rows;             // TMA box height: min(128, total rows)
   int tma_store;            // Z written through TMA stores (dense V layout, seq_len % 32 == 0)
+  unsigned long long* ts;   // trace slot or nullptr
 };
 
 template <int kDK>
@@ -99,7 +100,11 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
   using C = Cfg<kDK>;
   constexpr int kS = 0, kP = 128 * kNKB, kO = 192 * kNKB;
   constexpr uint32_t kCols = (kO + kDK) <= 256 ? 256u : 512u;
-  if (p.v_width && p.v_width[p.head_begin + blockIdx.y] == 0) return;   // every V feature of the head pruned
+  trace_cta_start(p.ts);
+  if (p.v_width && p.v_width[p.head_begin + blockIdx.y] == 0) {   // every V feature of the head pruned
+    trace_cta_end(p.ts);
+    return;
+  }
   extern __shared__ uint8_t smem_raw[];
   // 1024-byte aligned, derived from smem_raw by pointer arithmetic so the compiler keeps the shared
   // address space (an integer round trip would turn every access into a generic LD/ST)
@@ -463,6 +468,7 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
   tc_fence_before();
   __syncthreads();
   if (threadIdx.x == 0) ET_TLA(9);
+  trace_cta_end(p.ts);
   if (warp == 1) {
     __syncwarp();
     tc_fence_after();
@@ -517,6 +523,7 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   prm.dv_max = a.v_width_max;
   prm.scale_log2 = a.scale * kLog2e;
   prm.box_rows = (int)box_rows;
+  prm.ts = a.ts;
   // TMA stores of Z: dense per-head V, every 32-row group inside one sequence, Z 16-byte aligned
   prm.tma_store = (a.z_map == nullptr && a.v_width == nullptr && a.seq_len % 32 == 0 && rows >= 32 &&
                    aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;

@@ -54,7 +54,7 @@ __device__ __forceinline__ void st_act4(void* p, size_t idx, float4 v) {
 // All loads of the row are issued before any arithmetic so each warp has NCH * (NP + 2) 16/8-byte
 // requests in flight (the kernel is latency-bound otherwise).
 template <int NCH, int NP, int DT, int RT>
-__global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
+__device__ __forceinline__ void layernorm_row(const LnArgs& a) {
   const int row_i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (row_i >= a.M) return;
@@ -137,6 +137,16 @@ __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
                                  (v[c].z - mean) * rstd * gm.z + bt.z, (v[c].w - mean) * rstd * gm.w + bt.w);
     if (a.out_act) st_act4<DT>(a.out_act, row + col, y);
     if (a.out_resid) st_act4<RT>(a.out_resid, row + col, y);
+  }
+}
+
+template <int NCH, int NP, int DT, int RT>
+__global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
+  trace_cta_start(a.ts);
+  layernorm_row<NCH, NP, DT, RT>(a);
+  if (a.ts != nullptr) {
+    __syncthreads();
+    trace_cta_end(a.ts);
   }
 }
 

@@ -106,6 +106,7 @@ struct Params {
   void* Y;
   int ldy;
   long long part_stride;   // elements between split-K partial outputs (fp32 epilogue)
+  unsigned long long* ts;  // trace slot or nullptr
 };
 
 struct __align__(8) Barriers {
@@ -177,6 +178,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
 
   if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
+  trace_cta_start(p.ts);
   if (threadIdx.x == 0) ET_TL(0);
   if (threadIdx.x == 0) {
     for (int i = 0; i < kMaxKChunks; ++i) {
@@ -467,6 +469,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   tc_fence_before();
   __syncthreads();
   if (threadIdx.x == 0) ET_TL(500);
+  trace_cta_end(p.ts);
   if (warp == kWarpP) {
     __syncwarp();
     tc_fence_after();
@@ -580,6 +583,7 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   prm.Y = a.Y;
   prm.ldy = a.ldy;
   prm.part_stride = (long long)a.M * a.ldy;
+  prm.ts = a.ts;
   const int mblocks = (a.M + 127) / 128;
   int total_rows = 0;
   for (int s = 0; s < a.nseg; ++s) total_rows += a.seg[s].tile_rows;

@@ -371,4 +371,19 @@ __device__ __forceinline__ uint64_t fmul2(uint64_t a, uint64_t b) {
   return r;
 }
 
+
+// ------------------------------------------------------------------ device-side launch trace (et_trace_*)
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// thread 0 of every CTA: slot[0] = min start, slot[1] = ~max end (fire-and-forget reductions)
+__device__ __forceinline__ void trace_cta_start(unsigned long long* ts) {
+  if (ts != nullptr && threadIdx.x == 0) atomicMin(ts, globaltimer_ns());
+}
+__device__ __forceinline__ void trace_cta_end(unsigned long long* ts) {
+  if (ts != nullptr && threadIdx.x == 0) atomicMin(ts + 1, ~globaltimer_ns());
+}
+
 }  // namespace et
