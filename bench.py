@@ -182,9 +182,10 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------------------ roofline model
-def kernel_model(cfg, nnz: dict, kparts2: int, es: int, resid_es: int):
+def kernel_model(cfg, nnz: dict, kparts2: int, es: int, resid_es: int, ps: int):
     """Algorithmic bytes and (effective) FLOPs of ONE launch of each kernel kind for one layer of
-    `cfg`.  nnz: kept 16x16 tiles per matrix."""
+    `cfg`.  nnz: kept 16x16 tiles per matrix; ps: bytes per partial-sum
+    element handed to the LayerNorm kernels (2 on the FP16 path, 4 on BF16)."""
     M, d, f, H, S, B = cfg.tokens, cfg.d_model, cfg.d_ff, cfg.heads, cfg.seq_len, cfg.batch
     dk = d // H
     t = 512   # bytes per packed 16x16 fp16/bf16 tile
@@ -194,11 +195,11 @@ def kernel_model(cfg, nnz: dict, kparts2: int, es: int, resid_es: int):
         "qkv_gemm": (M * d * es + (nnz["wq"] + nnz["wk"] + nnz["wv"]) * t + M * 3 * d * es,
                      mm(nnz["wq"] + nnz["wk"] + nnz["wv"])),
         "attention": (M * 3 * d * es + M * d * es, 4.0 * pairs * dk),
-        "oproj_gemm": (M * d * es + nnz["wo"] * t + M * d * 4, mm(nnz["wo"])),
-        "ln1": (M * d * 4 + M * d * resid_es + M * d * es, 0.0),
+        "oproj_gemm": (M * d * es + nnz["wo"] * t + M * d * ps, mm(nnz["wo"])),
+        "ln1": (M * d * ps + M * d * resid_es + M * d * es, 0.0),
         "ffn1_gemm": (M * d * es + nnz["w1"] * t + M * f * es, mm(nnz["w1"])),
-        "ffn2_gemm": (M * f * es + nnz["w2"] * t + kparts2 * M * d * 4, mm(nnz["w2"])),
-        "ln2": (kparts2 * M * d * 4 + M * d * resid_es + M * d * resid_es, 0.0),
+        "ffn2_gemm": (M * f * es + nnz["w2"] * t + kparts2 * M * d * ps, mm(nnz["w2"])),
+        "ln2": (kparts2 * M * d * ps + M * d * resid_es + M * d * resid_es, 0.0),
     }
 
 
@@ -410,7 +411,7 @@ def our_arm(args):
         total_seqs = cfg.batch * world * K
         value = total_seqs / t_max
         es = 2
-        model = kernel_model(cfg, nnz_layers[0], layers[0].packed["w2"].c.kparts, es, es)
+        model = kernel_model(cfg, nnz_layers[0], layers[0].packed["w2"].c.kparts, es, es, 2 if dtype == "fp16" else 4)
         # dominant kernel: largest share of the traced step time
         tot = {k: sum(v) for k, v in per_kind.items()}
         dom = max(tot, key=tot.get) if tot else None

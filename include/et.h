@@ -139,19 +139,23 @@ et_status et_unpack(const et_packed_weight* w, void* dense_out, void* stream);
  *                      (the 1/sqrt(d_k) of Q moved before Q.K^T, line 159 §3.3)
  *   ET_EPI_BIAS_GELU / ET_EPI_BIAS_RELU  Y = act(acc + b)
  *   ET_EPI_F32         Y = acc (fp32, no bias) — partial sums for a LayerNorm epilogue
+ *   ET_EPI_PART16      Y = acc rounded to X's dtype (no bias) — 16-bit partial sums (FP16 path)
+ * ET_EPI_F32 / ET_EPI_PART16 with K > 768: Y is [ceil(K/768)][M, N], one split-K partial per plane.
  * X: [M, K] fp16/bf16, M % 128 == 0 not required (rows are masked).  b: [N] in X's dtype or NULL. */
-typedef enum { ET_EPI_BIAS = 0, ET_EPI_BIAS_SCALE = 1, ET_EPI_BIAS_GELU = 2, ET_EPI_BIAS_RELU = 3, ET_EPI_F32 = 4 } et_epilogue;
+typedef enum { ET_EPI_BIAS = 0, ET_EPI_BIAS_SCALE = 1, ET_EPI_BIAS_GELU = 2, ET_EPI_BIAS_RELU = 3, ET_EPI_F32 = 4,
+               ET_EPI_PART16 = 5 } et_epilogue;
 
 et_status et_linear_fwd(const et_packed_weight* w, const void* X, int32_t M, const void* bias, et_epilogue epi,
                         float scale, int32_t scale_cols, void* Y, void* stream);
 
 /* Residual + LayerNorm: out = LN(sum_p part[p] + bias + resid) * gamma + beta
- *   part: nparts x [M, N] fp32; bias [N] (dtype) or NULL; resid [M, N] in resid_dtype or NULL;
+ *   part: nparts x [M, N] in part_dtype (FP32, or dtype for 16-bit partials); bias [N] (dtype) or NULL; resid [M, N] in resid_dtype or NULL;
  *   gamma/beta fp32 [N]; out_act [M, N] in act_dtype (GEMM operand copy) and/or out_resid
  *   [M, N] in resid_dtype (either may be NULL).  Biased variance (reading C-11). */
-et_status et_layernorm_fwd(const float* part, int32_t nparts, int32_t M, int32_t N, const void* bias,
-                           et_dtype dtype, const void* resid, et_dtype resid_dtype, const float* gamma,
-                           const float* beta, float eps, void* out_act, void* out_resid, void* stream);
+et_status et_layernorm_fwd(const void* part, et_dtype part_dtype, int32_t nparts, int32_t M, int32_t N,
+                           const void* bias, et_dtype dtype, const void* resid, et_dtype resid_dtype,
+                           const float* gamma, const float* beta, float eps, void* out_act, void* out_resid,
+                           void* stream);
 
 /* ------------------------------------------------------------------------------------------
  * Attention descriptor.

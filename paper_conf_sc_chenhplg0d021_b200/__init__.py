@@ -22,7 +22,7 @@ FP16, BF16, FP32 = 0, 1, 2
 PRUNE_NONE, PRUNE_TILE, PRUNE_ROW, PRUNE_COL = 0, 1, 2, 3
 ATTN_AUTO, ATTN_SHORT, ATTN_LONG = 0, 1, 2
 ACT_GELU_ERF, ACT_RELU = 0, 1
-EPI_BIAS, EPI_BIAS_SCALE, EPI_BIAS_GELU, EPI_BIAS_RELU, EPI_F32 = 0, 1, 2, 3, 4
+EPI_BIAS, EPI_BIAS_SCALE, EPI_BIAS_GELU, EPI_BIAS_RELU, EPI_F32, EPI_PART16 = 0, 1, 2, 3, 4, 5
 
 _DT = {"fp16": FP16, "bf16": BF16, "fp32": FP32}
 _TORCH_DT = {FP16: torch.float16, BF16: torch.bfloat16, FP32: torch.float32}
@@ -86,7 +86,7 @@ _unpack = _sig("et_unpack", ctypes.c_int, [ctypes.POINTER(PackedWeightC), _vp, _
 _linear = _sig("et_linear_fwd", ctypes.c_int,
                [ctypes.POINTER(PackedWeightC), _vp, _i32, _vp, ctypes.c_int, _f32, _i32, _vp, _vp])
 _ln = _sig("et_layernorm_fwd", ctypes.c_int,
-           [_vp, _i32, _i32, _i32, _vp, ctypes.c_int, _vp, ctypes.c_int, _vp, _vp, _f32, _vp, _vp, _vp])
+           [_vp, ctypes.c_int, _i32, _i32, _i32, _vp, ctypes.c_int, _vp, ctypes.c_int, _vp, _vp, _f32, _vp, _vp, _vp])
 _short_max = _sig("et_attn_short_max", _i32, [_i32])
 
 SYMBOLS = ["et_last_error", "et_version", "et_prune_pack_query", "et_prune_pack", "et_unpack", "et_linear_fwd",
@@ -214,6 +214,8 @@ def linear_fwd(w: Packed, X: torch.Tensor, bias: torch.Tensor | None = None, epi
     if out is None:
         if epi == EPI_F32:
             out = torch.empty(w.c.kparts, M, N, dtype=torch.float32, device=X.device)
+        elif epi == EPI_PART16:
+            out = torch.empty(w.c.kparts, M, N, dtype=X.dtype, device=X.device)
         else:
             out = torch.empty(M, N, dtype=X.dtype, device=X.device)
     _check(_linear(ctypes.byref(w.c), X.data_ptr(), M, _ptr(bias), epi, scale, scale_cols, out.data_ptr(),
@@ -225,7 +227,7 @@ def layernorm_fwd(part: torch.Tensor, bias, resid, gamma, beta, eps: float, dtyp
                   out_act=None, out_resid=None, stream=None):
     """et_layernorm_fwd: LN(sum(part) + bias + resid)."""
     nparts, M, N = part.shape
-    _check(_ln(part.data_ptr(), nparts, M, N, _ptr(bias), dtype_code(dtype), _ptr(resid), dtype_code(resid_dtype),
+    _check(_ln(part.data_ptr(), dtype_code(part.dtype), nparts, M, N, _ptr(bias), dtype_code(dtype), _ptr(resid), dtype_code(resid_dtype),
                gamma.data_ptr(), beta.data_ptr(), eps, _ptr(out_act), _ptr(out_resid), _stream(stream)))
     return out_act, out_resid
 

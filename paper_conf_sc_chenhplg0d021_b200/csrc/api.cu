@@ -255,12 +255,14 @@ et_status et_linear_fwd(const et_packed_weight* w, const void* X, int32_t M, con
   return gemm_run(a, static_cast<cudaStream_t>(stream));
 }
 
-et_status et_layernorm_fwd(const float* part, int32_t nparts, int32_t M, int32_t N, const void* bias,
-                           et_dtype dtype, const void* resid, et_dtype resid_dtype, const float* gamma,
-                           const float* beta, float eps, void* out_act, void* out_resid, void* stream) {
+et_status et_layernorm_fwd(const void* part, et_dtype part_dtype, int32_t nparts, int32_t M, int32_t N,
+                           const void* bias, et_dtype dtype, const void* resid, et_dtype resid_dtype,
+                           const float* gamma, const float* beta, float eps, void* out_act, void* out_resid,
+                           void* stream) {
   if (!part || nparts < 1 || (gamma == nullptr) != (beta == nullptr))
     return fail(ET_ERR_INVALID_ARG, "et_layernorm_fwd: bad arguments");
-  LnArgs a{part, nparts, M, N, bias, dtype, resid, resid_dtype, gamma, beta, eps, out_act, out_resid};
+  LnArgs a{part, nparts, M, N, bias, dtype, resid, resid_dtype, gamma, beta, eps, out_act, out_resid, nullptr,
+           part_dtype};
   return layernorm_run(a, static_cast<cudaStream_t>(stream));
 }
 

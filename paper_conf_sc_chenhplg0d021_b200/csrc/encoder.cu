@@ -27,6 +27,12 @@ struct Carver {
   }
 };
 
+// Precision of the O-projection / FFN2 partial sums handed to the LayerNorm kernel: FP16 storage
+// on the FP16 path ("pure FP16"; reading C-9 — accumulation stays FP32
+// in TMEM), FP32 on the BF16 path (8-bit mantissa partials would cost accuracy).
+et_dtype part_dtype_of(et_dtype dt) { return dt == ET_FP16 ? ET_FP16 : ET_FP32; }
+et_epilogue part_epi_of(et_dtype dt) { return dt == ET_FP16 ? ET_EPI_PART16 : ET_EPI_F32; }
+
 bool long_form_for(const et_attn_desc* d) {
   const int dk = d->d_model / d->heads;
   if (d->mode == ET_ATTN_LONG) return true;
@@ -80,7 +86,7 @@ struct BlockWs {
   void* qkv;        // [M, ldq]
   int ldq;
   void* z;          // [M, d]
-  float* part;      // [kparts_max][M, d]
+  void* part;       // [kparts_max][M, d] partial sums (part_dtype_of)
   int32_t* v_col;   // [H]   (attention-aware only)
   int32_t* v_width; // [H]
   void* bv_packed;  // [vmax]
@@ -97,7 +103,7 @@ void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, Blo
   ws->ldq = 2 * d->d_model + vmax;
   ws->qkv = c.take(M * ws->ldq * es);
   ws->z = c.take(M * d->d_model * es);
-  ws->part = static_cast<float*>(c.take((size_t)kparts_max * M * d->d_model * 4));
+  ws->part = c.take((size_t)kparts_max * M * d->d_model * 4);   // sized for FP32
   ws->v_col = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
   ws->v_width = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
   ws->bv_packed = c.take((size_t)vmax * es);
@@ -178,7 +184,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   o.seg[0] = seg_of(wo, nullptr, 0);
   o.Y = ws.part;
   o.ldy = dm;
-  o.epi = ET_EPI_F32;
+  o.epi = part_epi_of(d->dtype);
   o.ts = trace_slot(ET_K_OPROJ);
   return gemm_run(o, st);
 }
@@ -257,7 +263,7 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   ET_TRY(run_attention_block(desc, X, wq, wk, wv, wo, bq, bk, bv, bo, ws, &bo_eff, st));
   const int M = desc->batch * desc->seq_len;
   LnArgs ln{ws.part, 1, M, dm, bo_eff, desc->dtype, ln_gamma ? X : nullptr, desc->dtype, ln_gamma, ln_beta, ln_eps,
-            out, nullptr, nullptr};
+            out, nullptr, nullptr, part_dtype_of(desc->dtype)};
   ln.ts = trace_slot(ET_K_LN1);
   ET_TRY(layernorm_run(ln, st));   // gamma == NULL: out = attn = part + b_O' (no residual, no LN)
   return ET_OK;
@@ -346,7 +352,7 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     ET_TRY(run_attention_block(desc, cur_act, &L.wq, &L.wk, &L.wv, &L.wo, L.bq, L.bk, L.bv, L.bo, ws, &bo_eff, st));
     // 4. Y1 = LN(X + attn)
     LnArgs ln1{ws.part, 1, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,
-               y1a, split ? y1r : nullptr, nullptr};
+               y1a, split ? y1r : nullptr, nullptr, part_dtype_of(desc->dtype)};
     ln1.ts = trace_slot(ET_K_LN1);
     ET_TRY(layernorm_run(ln1, st));
     // 5. U = act(Y1 W1'^T + b1)
@@ -374,12 +380,12 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     f2.seg[0] = seg_of(&L.w2, nullptr, 0);
     f2.Y = ws.part;
     f2.ldy = dm;
-    f2.epi = ET_EPI_F32;
+    f2.epi = part_epi_of(desc->dtype);
     f2.ts = trace_slot(ET_K_FFN2);
     ET_TRY(gemm_run(f2, st));
     // 7. Y2 = LN(Y1 + F + b2)
     LnArgs ln2{ws.part, L.w2.kparts, (int)M, dm, L.b2, desc->dtype, y1r, resid_dtype, L.ln2_g, L.ln2_b, ln_eps,
-               split ? next_act : nullptr, next_res, nullptr};
+               split ? next_act : nullptr, next_res, nullptr, part_dtype_of(desc->dtype)};
     ln2.ts = trace_slot(ET_K_LN2);
     ET_TRY(layernorm_run(ln2, st));
     cur_res = next_res;

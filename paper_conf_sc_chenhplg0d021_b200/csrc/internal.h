@@ -2,6 +2,7 @@
 // launch wrappers (kernels/*.cu).  Not part of the public ABI.
 #pragma once
 #include <cuda_runtime.h>
+#include <utility>
 #include <cstdarg>
 #include <cstdint>
 #include <cstddef>
@@ -75,7 +76,7 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream);
 
 // ---------------------------------------------------------------- LayerNorm (kernels/layernorm.cu)
 struct LnArgs {
-  const float* part;
+  const void* part;         // [nparts][M][N] partial sums in part_dtype (FP32 or the operand dtype)
   int nparts, M, N;
   const void* bias;
   et_dtype dtype;
@@ -87,6 +88,7 @@ struct LnArgs {
   void* out_act;
   void* out_resid;
   unsigned long long* ts;   // trace slot or nullptr
+  et_dtype part_dtype;
 };
 et_status layernorm_run(const LnArgs& a, cudaStream_t stream);
 
@@ -131,7 +133,25 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream);
 
 // ---------------------------------------------------------------- tracing (api.cu)
 // Record a mark of `kind` on `stream` if tracing is enabled; counts one kernel launch.
-unsigned long long* trace_slot(int kind);   // device slot of the next traced launch, or nullptr
+unsigned long long* trace_slot(int kind);
+
+// Launch with programmatic stream serialisation (PDL): the kernel may begin while the previous
+// kernel on the stream finishes; it must call pdl_wait() (ptx.cuh) before touching global data.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
+                       Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}   // device slot of the next traced launch, or nullptr
 void count_launch();
 void add_launches(long long n);
 long long launch_count();

@@ -100,6 +100,8 @@ __global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant
   using C = Cfg<kDK>;
   constexpr int kS = 0, kP = 128 * kNKB, kO = 192 * kNKB;
   constexpr uint32_t kCols = (kO + kDK) <= 256 ? 256u : 512u;
+  pdl_trigger();
+  pdl_wait();   // QKV (and the attention-aware head tables) of the predecessors are visible from here
   trace_cta_start(p.ts);
   if (p.v_width && p.v_width[p.head_begin + blockIdx.y] == 0) {   // every V feature of the head pruned
     trace_cta_end(p.ts);
@@ -484,9 +486,8 @@ et_status launch(const CUtensorMap& tm, const CUtensorMap& tz, const AParams& pr
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [&] { attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); });
   ET_CUDA(attr_err);
-  kern<<<grid, kThreads, smem, stream>>>(tm, tz, prm);
+  ET_CUDA(launch_pdl(kern, grid, dim3(kThreads), smem, stream, tm, tz, prm));
   count_launch();
-  ET_CUDA(cudaGetLastError());
   return ET_OK;
 }
 

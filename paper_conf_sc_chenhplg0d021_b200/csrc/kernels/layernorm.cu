@@ -53,7 +53,7 @@ __device__ __forceinline__ void st_act4(void* p, size_t idx, float4 v) {
 // One warp per row; NCH = ceil(N / 128) chunks of 4 columns per lane, NP split-K partial inputs.
 // All loads of the row are issued before any arithmetic so each warp has NCH * (NP + 2) 16/8-byte
 // requests in flight (the kernel is latency-bound otherwise).
-template <int NCH, int NP, int DT, int RT>
+template <int NCH, int NP, int DT, int RT, bool P16>
 __device__ __forceinline__ void layernorm_row(const LnArgs& a) {
   const int row_i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
@@ -67,7 +67,7 @@ __device__ __forceinline__ void layernorm_row(const LnArgs& a) {
   // destination first and serialise the row's loads behind each other's latency.
   const bool has_bias = a.bias != nullptr, has_res = a.resid != nullptr;
   const void* bias_p = has_bias ? a.bias : a.part;
-  const void* res_p = has_res ? a.resid : a.part;
+  const void* res_p = has_res ? a.resid : a.part;   // (dummy addresses: masked below)
 #pragma unroll
   for (int c = 0; c < NCH; ++c) ok[c] = c * 128 + lane * 4 < a.N;
 #pragma unroll
@@ -75,7 +75,15 @@ __device__ __forceinline__ void layernorm_row(const LnArgs& a) {
     const int col = ok[c] ? c * 128 + lane * 4 : 0;
 #pragma unroll
     for (int q = 0; q < NP; ++q)
-      part[q][c] = __ldcs(reinterpret_cast<const float4*>(a.part + (size_t)q * a.M * a.N + row + col));
+      if constexpr (P16) {   // 16-bit partial sums in the operand dtype (FP16 path, reading C-9)
+        const uint2 u = __ldcs(reinterpret_cast<const uint2*>(static_cast<const uint16_t*>(a.part) +
+                                                               (size_t)q * a.M * a.N + row + col));
+        const float2 lo = unpack2<DT == ET_BF16>(u.x), hi = unpack2<DT == ET_BF16>(u.y);
+        part[q][c] = make_float4(lo.x, lo.y, hi.x, hi.y);
+      } else {
+        part[q][c] = __ldcs(reinterpret_cast<const float4*>(static_cast<const float*>(a.part) +
+                                                            (size_t)q * a.M * a.N + row + col));
+      }
     bias[c] = ld_act4<DT>(bias_p, has_bias ? col : 0);
     res[c] = ld_act4<RT>(res_p, has_res ? row + col : 0);
   }
@@ -140,39 +148,49 @@ __device__ __forceinline__ void layernorm_row(const LnArgs& a) {
   }
 }
 
-template <int NCH, int NP, int DT, int RT>
+template <int NCH, int NP, int DT, int RT, bool P16>
 __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
+  pdl_trigger();
+  pdl_wait();
   trace_cta_start(a.ts);
-  layernorm_row<NCH, NP, DT, RT>(a);
+  layernorm_row<NCH, NP, DT, RT, P16>(a);
   if (a.ts != nullptr) {
     __syncthreads();
     trace_cta_end(a.ts);
   }
 }
 
-template <int NCH, int DT, int RT>
+template <int NCH, int DT, int RT, bool P16>
 et_status launch_np(const LnArgs& a, cudaStream_t stream) {
   const int threads = 128;
   const int blocks = (a.M * 32 + threads - 1) / threads;
+  cudaError_t e = cudaSuccess;
   switch (a.nparts) {
-    case 1: layernorm_kernel<NCH, 1, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
-    case 2: layernorm_kernel<NCH, 2, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
-    case 3: layernorm_kernel<NCH, 3, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
-    case 4: layernorm_kernel<NCH, 4, DT, RT><<<blocks, threads, 0, stream>>>(a); break;
+    case 1: e = launch_pdl(layernorm_kernel<NCH, 1, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
+    case 2: e = launch_pdl(layernorm_kernel<NCH, 2, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
+    case 3: e = launch_pdl(layernorm_kernel<NCH, 3, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
+    case 4: e = launch_pdl(layernorm_kernel<NCH, 4, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
     default: return fail(ET_ERR_UNSUPPORTED, "LayerNorm: up to 4 partial inputs (got %d)", a.nparts);
   }
+  ET_CUDA(e);
   count_launch();
-  ET_CUDA(cudaGetLastError());
   return ET_OK;
 }
 
 template <int NCH>
 et_status launch_dt(const LnArgs& a, cudaStream_t stream) {
   const int dt = a.dtype, rt = a.resid ? a.resid_dtype : (a.out_resid ? a.resid_dtype : a.dtype);
-  if (dt == ET_FP16 && rt == ET_FP16) return launch_np<NCH, ET_FP16, ET_FP16>(a, stream);
-  if (dt == ET_FP16 && rt == ET_FP32) return launch_np<NCH, ET_FP16, ET_FP32>(a, stream);
-  if (dt == ET_BF16 && rt == ET_BF16) return launch_np<NCH, ET_BF16, ET_BF16>(a, stream);
-  if (dt == ET_BF16 && rt == ET_FP32) return launch_np<NCH, ET_BF16, ET_FP32>(a, stream);
+  if (a.part_dtype != ET_FP32 && a.part_dtype != a.dtype)
+    return fail(ET_ERR_UNSUPPORTED, "LayerNorm: partial sums must be FP32 or the operand dtype");
+  const bool p16 = a.part_dtype != ET_FP32;
+  if (dt == ET_FP16 && rt == ET_FP16)
+    return p16 ? launch_np<NCH, ET_FP16, ET_FP16, true>(a, stream) : launch_np<NCH, ET_FP16, ET_FP16, false>(a, stream);
+  if (dt == ET_FP16 && rt == ET_FP32)
+    return p16 ? launch_np<NCH, ET_FP16, ET_FP32, true>(a, stream) : launch_np<NCH, ET_FP16, ET_FP32, false>(a, stream);
+  if (dt == ET_BF16 && rt == ET_BF16)
+    return p16 ? launch_np<NCH, ET_BF16, ET_BF16, true>(a, stream) : launch_np<NCH, ET_BF16, ET_BF16, false>(a, stream);
+  if (dt == ET_BF16 && rt == ET_FP32)
+    return p16 ? launch_np<NCH, ET_BF16, ET_FP32, true>(a, stream) : launch_np<NCH, ET_BF16, ET_FP32, false>(a, stream);
   return fail(ET_ERR_UNSUPPORTED, "LayerNorm: dtype pair (%d, %d) not supported", dt, rt);
 }
 

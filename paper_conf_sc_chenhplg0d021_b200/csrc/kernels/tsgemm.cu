@@ -109,11 +109,11 @@ struct Params {
   unsigned long long* ts;  // trace slot or nullptr
 };
 
-struct __align__(8) Barriers {
+struct __align__(16) Barriers {
   // single-use barriers per A chunk / tile chunk (a warp may run laps ahead of a slot's reuse, and a
   // parity wait on a reused barrier cannot tell those phases apart)
-  uint64_t xfull[kMaxKChunks];   // A chunk j landed in its slot (TMA transaction bytes)
-  uint64_t xfree[kMaxKChunks];   // A chunk j read out of its slot (4 fill warps)
+  uint64_t xfull[kMaxKChunks];   // A load #s landed in its slot (TMA transaction bytes)
+  uint64_t xfree[kMaxKChunks];   // A load #s read out of its slot (4 fill warps)
   uint64_t afill[kMaxKChunks];   // A chunk j stored into TMEM (4 fill warps)
   uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
   uint64_t bfull[kMaxBChunks];
@@ -152,6 +152,9 @@ __device__ __forceinline__ void gelu_erf2(float& x0, float& x1) {
   x1 = g.y;
 }
 
+// epilogues that write raw accumulators (no bias) as split-K partial planes [kparts][M][ldy]
+constexpr bool is_partial(int e) { return e == ET_EPI_F32 || e == ET_EPI_PART16; }
+
 template <int kEpi, bool kBF16>
 __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
                                                              const __grid_constant__ CUtensorMap tmap_y,
@@ -178,7 +181,10 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
 
   if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
-  trace_cta_start(p.ts);
+  // A chunks are loaded in a rotated order: the CTAs of one token block (its pieces) start a quarter
+  // of the block apart, so they do not all hit the same L2 lines at the same moment.
+  const int a_rot = (blockIdx.x & 3) * (nk >> 2);
+  auto a_chunk = [&](int sq) { return sq + a_rot < nk ? sq + a_rot : sq + a_rot - nk; };
   if (threadIdx.x == 0) ET_TL(0);
   if (threadIdx.x == 0) {
     for (int i = 0; i < kMaxKChunks; ++i) {
@@ -195,9 +201,12 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     fence_mbar_init();
   }
   if (warp == kWarpP) tmem_alloc<512>(&bar.tmem_base);
+  pdl_trigger();
+  pdl_wait();   // the predecessor's output (A, and a bias it may have produced) is visible from here
+  trace_cta_start(p.ts);
   // stage the per-CTA metadata once (one global round trip instead of one per tile row)
   for (int i = threadIdx.x; i <= nrows; i += blockDim.x) bar.rptr[i] = rp[pc.i0 + i] - pb;
-  if constexpr (kEpi != ET_EPI_F32) {
+  if constexpr (!is_partial(kEpi)) {
     const uint32_t* bsrc = static_cast<const uint32_t*>(sg.bias);
     for (int i = threadIdx.x; i < nrows * 8; i += blockDim.x)
       bar.bias_s[i] = bsrc ? __ldg(bsrc + (size_t)pc.i0 * 8 + i) : 0u;
@@ -217,9 +226,10 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     const int rr = q * 32 + lane;
     const uint32_t tq = tbase + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
-    for (int j = warp >> 2; j < nk; j += kFillSets) {
-      mbar_wait_warp(&bar.xfull[j], 0);
-      const uint8_t* rowp = ring + (j % kSlots) * kSlotBytes + rr * 128;
+    for (int sq = warp >> 2; sq < nk; sq += kFillSets) {   // load sequence position sq holds chunk j
+      const int j = a_chunk(sq);
+      mbar_wait_warp(&bar.xfull[sq], 0);
+      const uint8_t* rowp = ring + (sq % kSlots) * kSlotBytes + rr * 128;
       uint32_t v[32];
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
@@ -227,12 +237,13 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         v[4 * c] = u.x; v[4 * c + 1] = u.y; v[4 * c + 2] = u.z; v[4 * c + 3] = u.w;
       }
       __syncwarp();
-      if (lane == 0) mbar_arrive(&bar.xfree[j]);   // the producer may reuse the slot
+      if (lane == 0) mbar_arrive(&bar.xfree[sq]);   // the producer may reuse the slot
       tmem_st32(tq + j * 32, v);
       tmem_st_wait();
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&bar.afill[j]);
+      if (lane == 0 && q == 0) ET_TL(2 + sq);
     }
   }
 
@@ -268,7 +279,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         uint8_t* dst = ring + slot * kSlotBytes;
         if (s < nk) {
           mbar_expect_tx(&bar.xfull[s], p.box_rows * 128);
-          tma_load_2d(dst, &tmap_x, &bar.xfull[s], kx0 + s * 64, m0);
+          tma_load_2d(dst, &tmap_x, &bar.xfull[s], kx0 + a_chunk(s) * 64, m0);
         } else {
           const int c = s - nk;
           const int nt = min(kChunkTiles, pe - pb - c * kChunkTiles);
@@ -389,7 +400,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           // a row with no kept tile was never written: its accumulator is zero (output = epi(bias))
           float x0 = empty_row ? 0.0f : __uint_as_float(r[a * 16 + c]);
           float x1 = empty_row ? 0.0f : __uint_as_float(r[a * 16 + c + 1]);
-          if constexpr (kEpi != ET_EPI_F32) {
+          if constexpr (!is_partial(kEpi)) {
             const float2 bb = unpack2<kBF16>(bar.bias_s[t * 8 + c / 2]);
             uint64_t xx = fadd2(f2pk(x0, x1), f2pk(bb.x, bb.y));
             if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
@@ -437,7 +448,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         fence_proxy_async_smem();
         __syncwarp();
         if (lane == 0) {
-          if constexpr (kEpi == ET_EPI_F32) tma_store_3d(&tmap_y, st, col0, row0, z);
+          if constexpr (is_partial(kEpi)) tma_store_3d(&tmap_y, st, col0, row0, z);
           else tma_store_2d(&tmap_y, st, col0, row0);
           bulk_commit_group();
         }
@@ -452,7 +463,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
             for (int c = 0; c < 16; c += 4)
               *reinterpret_cast<float4*>(y + c) = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
           } else {
-            uint16_t* y = static_cast<uint16_t*>(p.Y) + (size_t)row * p.ldy + col0;
+            uint16_t* y = static_cast<uint16_t*>(p.Y) + (kEpi == ET_EPI_PART16 ? (size_t)z * p.part_stride : 0) +
+                          (size_t)row * p.ldy + col0;
             *reinterpret_cast<uint4*>(y) = make_uint4(pack2<kBF16>(v[0], v[1]), pack2<kBF16>(v[2], v[3]),
                                                       pack2<kBF16>(v[4], v[5]), pack2<kBF16>(v[6], v[7]));
             *reinterpret_cast<uint4*>(y + 8) = make_uint4(pack2<kBF16>(v[8], v[9]), pack2<kBF16>(v[10], v[11]),
@@ -505,9 +517,8 @@ et_status launch_typed(const CUtensorMap& tm, const CUtensorMap& tmy, const Para
     attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   });
   ET_CUDA(attr_err);
-  kern<<<grid, kThreads, kSmemBytes, stream>>>(tm, tmy, prm);
+  ET_CUDA(launch_pdl(kern, grid, dim3(kThreads), kSmemBytes, stream, tm, tmy, prm));
   count_launch();
-  ET_CUDA(cudaGetLastError());
   return ET_OK;
 }
 
@@ -546,16 +557,21 @@ et_status make_tmap_2d_sw64(CUtensorMap* tm, const void* base, et_dtype dtype, u
   return ET_OK;
 }
 
-et_status make_tmap_3d_f32(CUtensorMap* tm, void* base, uint64_t cols, uint64_t rows, uint64_t planes,
-                           uint32_t box_cols, uint32_t box_rows) {
+// [planes][rows][cols] tensor (fp32: SWIZZLE_128B, box 32 cols = 128 B; 16-bit: SWIZZLE_64B, 32 cols = 64 B)
+et_status make_tmap_3d(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t cols, uint64_t rows, uint64_t planes,
+                       uint32_t box_cols, uint32_t box_rows) {
   EncodeTiledFn enc = get_encode();
   if (!enc) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  const uint64_t es = dtype_size(dtype);
   cuuint64_t dims[3] = {cols, rows, planes};
-  cuuint64_t strides[2] = {cols * 4, cols * rows * 4};
+  cuuint64_t strides[2] = {cols * es, cols * rows * es};
   cuuint32_t box[3] = {box_cols, box_rows, 1};
   cuuint32_t estr[3] = {1, 1, 1};
-  CUresult r = enc(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, base, dims, strides, box, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+  CUtensorMapDataType dt = dtype == ET_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                           : dtype == ET_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                              : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
+  CUresult r = enc(tm, dt, 3, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   es == 4 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled (3d) failed (%d)", (int)r);
   return ET_OK;
@@ -567,8 +583,8 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   if (!aligned16(a.X) || (a.ldx * 2) % 16 || (a.k0 * 2) % 16)
     return fail(ET_ERR_INVALID_ARG, "tile GEMM: X must be 16-byte aligned with 16-byte row pitch");
   const int kparts = (a.K + 767) / 768;
-  if (kparts > 1 && a.epi != ET_EPI_F32)
-    return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K > 768 needs the fp32 split-K epilogue");
+  if (kparts > 1 && a.epi != ET_EPI_F32 && a.epi != ET_EPI_PART16)
+    return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K > 768 needs a partial-sum (split-K) epilogue");
   if (a.M <= 0) return ET_OK;
 
   Params prm{};
@@ -638,9 +654,9 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   // output tensor map: [M, ldy] in the operand dtype, box 32 cols x 32 rows (one epilogue warp's
   // staging tile, SWIZZLE_64B); fp32 partials: [kparts, M, ldy], box 32 x 32 x 1 (SWIZZLE_128B).
   CUtensorMap tmy;
-  if (a.epi == ET_EPI_F32) {
-    ET_TRY(make_tmap_3d_f32(&tmy, a.Y, (uint64_t)a.ldy, (uint64_t)a.M, (uint64_t)kparts, 32,
-                            a.M < 32 ? (uint32_t)a.M : 32u));
+  if (a.epi == ET_EPI_F32 || a.epi == ET_EPI_PART16) {
+    ET_TRY(make_tmap_3d(&tmy, a.Y, a.epi == ET_EPI_F32 ? ET_FP32 : a.dtype, (uint64_t)a.ldy, (uint64_t)a.M,
+                        (uint64_t)kparts, 32, a.M < 32 ? (uint32_t)a.M : 32u));
   } else {
     ET_TRY(make_tmap_2d_sw64(&tmy, a.Y, a.dtype, (uint64_t)a.M, (uint64_t)a.ldy, (uint64_t)a.ldy, 32,
                              a.M < 32 ? (uint32_t)a.M : 32u));
@@ -658,6 +674,8 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
                                      : launch_typed<ET_EPI_BIAS_RELU, false>(tm, tmy, prm, grid, stream);
     case ET_EPI_F32: return bf ? launch_typed<ET_EPI_F32, true>(tm, tmy, prm, grid, stream)
                                : launch_typed<ET_EPI_F32, false>(tm, tmy, prm, grid, stream);
+    case ET_EPI_PART16: return bf ? launch_typed<ET_EPI_PART16, true>(tm, tmy, prm, grid, stream)
+                                  : launch_typed<ET_EPI_PART16, false>(tm, tmy, prm, grid, stream);
   }
   return fail(ET_ERR_INVALID_ARG, "tile GEMM: bad epilogue %d", (int)a.epi);
 }

@@ -386,4 +386,12 @@ __device__ __forceinline__ void trace_cta_end(unsigned long long* ts) {
   if (ts != nullptr && threadIdx.x == 0) atomicMin(ts + 1, ~globaltimer_ns());
 }
 
+// ------------------------------------------------------------------ programmatic dependent launch
+// Every forward kernel is launched with programmatic stream serialisation (launch_pdl): it may start
+// while its predecessor drains, does only private setup (barriers, TMEM, smem carving) before
+// pdl_wait(), and reads / writes no global data before it.  pdl_trigger() lets the successor launch
+// (it is scheduled once every CTA of this grid has triggered or exited).
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 }  // namespace et

@@ -83,6 +83,24 @@ def test_linear_fp32_partials_split_k(etm, K):
     assert np.abs(g - ref).max() <= 1e-5 * max(1.0, np.abs(ref).max())
 
 
+@pytest.mark.parametrize("K,M", [(768, 384), (3072, 300)])
+def test_linear_fp16_partials_split_k(etm, K, M):
+    """ET_EPI_PART16: each split-K plane is the FP32 accumulator rounded once to FP16; the planes sum
+    to X . W'^T within the per-plane rounding bound (the FP16 path's O-proj / FFN2 partial sums)."""
+    dtype, N = "fp16", 768
+    Wnp = make_matrix(32, (N, K), 0.02, dtype)
+    X = make_matrix(33, (M, K), 1.0, dtype)
+    pk = etm.prune_pack(dev_tensor(Wnp, dtype), "tile", 0.8)
+    P = etm.linear_fwd(pk, dev_tensor(X, dtype), None, etm.EPI_PART16)
+    torch.cuda.synchronize()
+    assert P.dtype == torch.float16 and P.shape == (K // 768, M, N)
+    Wp = op.prune_tile(Wnp, 0.8)["W_pruned"]
+    g = P.double().cpu().numpy()
+    for z in range(K // 768):   # each plane: its K part's exact product, rounded to fp16 once
+        ref = oe.linear(X[:, z * 768:(z + 1) * 768], Wp[:, z * 768:(z + 1) * 768], None)
+        assert np.all(np.abs(g[z] - ref) <= _rounding_bound(ref, dtype) + 1e-5)
+
+
 def test_pruned_tile_values_do_not_matter_bitexact(etm):
     """P5: same mask, different values inside pruned tiles => bit-identical output."""
     dtype, M, d = "fp16", 256, 768
