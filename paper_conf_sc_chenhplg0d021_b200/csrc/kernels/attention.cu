@@ -94,7 +94,7 @@ __device__ __forceinline__ void tmem_alloc_n(uint32_t* slot) { tmem_alloc<kCols>
 // kNKB: score blocks resident in TMEM (short form: 1 => seq_len <= 128, 2 => <= 256; long form: the
 // two S buffers).  TMEM: S [0, 128 kNKB), P [128 kNKB, 192 kNKB), O [192 kNKB, 192 kNKB + kDK).
 template <bool kBF16, int kDK, bool kLong, int kNKB>
-__global__ void __launch_bounds__(kThreads, 1) attn_kernel(const __grid_constant__ CUtensorMap tmap,
+__global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __grid_constant__ CUtensorMap tmap,
                                                            const __grid_constant__ CUtensorMap tmap_z,
                                                            const __grid_constant__ AParams p) {
   using C = Cfg<kDK>;
