@@ -9,7 +9,7 @@
 //     With A in shared memory every N=16 MMA re-reads 4 KB of A and the kernel is capped near 20 %
 //     of peak by smem bandwidth.  Fill: TMA (SWIZZLE_128B) -> smem -> registers of the 24 MMA /
 //     epilogue warps (idle during the prologue) -> tcgen05.st.
-//   * one unified 9-slot shared-memory ring carries first the A chunks (all in flight at once: the
+//   * one unified shared-memory ring (9 or 11 slots of 16 KB) carries first the A chunks (all in flight at once: the
 //     prologue is bound by L2 bandwidth, not by ring depth) and then the packed tiles (512 B each,
 //     contiguous per (K part, tile row), 1-D bulk copies of 32 tiles + their column indices).
 //   * 8 MMA warps, one accumulator (16 TMEM columns) each, so 8 independent accumulation chains are
@@ -59,14 +59,12 @@ __device__ __forceinline__ unsigned long long gtime() {
 namespace {
 
 constexpr int kMaxPieces = 64;
-#ifndef ET_GEMM_SLOTS
-#define ET_GEMM_SLOTS 9
-#endif
+
 // Unified staging ring: the A chunks of the K part (128 rows x 64 K, SWIZZLE_128B) come first in the
 // load sequence, then the tile chunks (32 packed tiles each).  Every A load is in flight at once during
 // the prologue (the whole ring is free then), and the slots are reused for tiles as soon as the
 // fill warps have moved their A chunk into TMEM.
-constexpr int kSlots = ET_GEMM_SLOTS;
+constexpr int kMaxSlots = 11;
 constexpr int kSlotBytes = 16384;
 constexpr int kChunkTiles = 32;  // tiles per tile chunk (16 KB)
 constexpr int kMaxKChunks = 12;  // K <= 768 per part
@@ -117,17 +115,24 @@ struct __align__(16) Barriers {
   uint64_t afill[kMaxKChunks];   // A chunk j stored into TMEM (4 fill warps)
   uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
   uint64_t bfull[kMaxBChunks];
-  alignas(16) int tcol[kSlots][kChunkTiles + 4];   // bulk-copy destination (16-byte aligned): tile columns
+  alignas(16) int tcol[kMaxSlots][kChunkTiles + 4];   // bulk-copy destination (16-byte aligned): tile columns
   int rptr[kMaxRows + 1];        // this CTA's row pointers, relative to its first tile
   uint32_t bias_s[kMaxRows * 8]; // this CTA's bias slice (16-bit pairs)
   uint32_t tmem_base;
   int rows_seen[kEpiGroups];     // per epilogue group: rows whose MMAs were observed complete (in order)
 };
 
-constexpr size_t kSmemRing = (size_t)kSlots * kSlotBytes;
-constexpr size_t kSmemStage = (size_t)kEpiWarps * 4096;   // 32 rows x 128 B per epilogue warp
-constexpr size_t kSmemBytes = 1024 + kSmemRing + kSmemStage + sizeof(Barriers);
-static_assert(kSmemBytes <= 232448, "shared memory budget");
+// Per epilogue: staging per epilogue warp (32 rows x 32 columns: 128 B rows in FP32, 64 B in 16-bit)
+// and as many ring slots as the rest of the 227 KB allows (9 with FP32 staging, 11 with 16-bit).
+template <int kEpi> struct Smem {
+  static constexpr size_t kStageWarp = kEpi == ET_EPI_F32 ? 4096 : 2048;
+  static constexpr size_t kStage = (size_t)kEpiWarps * kStageWarp;
+  static constexpr int kSlots = kEpi == ET_EPI_F32 ? 9 : 11;
+  static constexpr size_t kRing = (size_t)kSlots * kSlotBytes;
+  static constexpr size_t kBytes = 1024 + kRing + kStage + sizeof(Barriers);
+  static_assert(kBytes <= 232448, "shared memory budget");
+  static_assert(kSlots <= kMaxSlots, "slot metadata");
+};
 
 // GELU(x) = x Phi(x) = 0.5 x (1 + erf(x / sqrt 2)) (reading C-12), evaluated as
 //   GELU(x) = max(x, 0) - |x| e,   e = 0.5 erfc(t) = 2^(-g(t) - 1),   t = |x| / sqrt 2 (clamped to 4)
@@ -164,8 +169,10 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   // address space (an integer round trip would turn every access into a generic LD/ST)
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* ring = smem;
-  uint8_t* sStage = smem + kSmemRing;
-  Barriers& bar = *reinterpret_cast<Barriers*>(smem + kSmemRing + kSmemStage);
+  using SM = Smem<kEpi>;
+  constexpr int kSlots = SM::kSlots;
+  uint8_t* sStage = smem + SM::kRing;
+  Barriers& bar = *reinterpret_cast<Barriers*>(smem + SM::kRing + SM::kStage);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -201,16 +208,12 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     fence_mbar_init();
   }
   if (warp == kWarpP) tmem_alloc<512>(&bar.tmem_base);
-  pdl_trigger();
-  pdl_wait();   // the predecessor's output (A, and a bias it may have produced) is visible from here
-  trace_cta_start(p.ts);
-  // stage the per-CTA metadata once (one global round trip instead of one per tile row)
+  // stage the per-CTA row pointers once (static weight metadata, not written by any predecessor, so
+  // this overlaps the previous kernel's tail under PDL).  Everything the predecessor produces (A,
+  // and a bias it may have computed) is read only after pdl_wait(): by the producer before its
+  // first load and by the epilogue warps before they stage the bias.
   for (int i = threadIdx.x; i <= nrows; i += blockDim.x) bar.rptr[i] = rp[pc.i0 + i] - pb;
-  if constexpr (!is_partial(kEpi)) {
-    const uint32_t* bsrc = static_cast<const uint32_t*>(sg.bias);
-    for (int i = threadIdx.x; i < nrows * 8; i += blockDim.x)
-      bar.bias_s[i] = bsrc ? __ldg(bsrc + (size_t)pc.i0 * 8 + i) : 0u;
-  }
+  pdl_trigger();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -255,6 +258,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     // never waits for a row that itself needs the chunk being loaded.
     if (lane == 0) {
       tma_prefetch_desc(&tmap_x);
+      pdl_wait();
+      if (p.ts != nullptr) atomicMin(p.ts, globaltimer_ns());   // trace: this CTA's work starts
       const int kx0 = z * p.Kp;
       const uint8_t* vals = sg.values + (size_t)pb * 512;
       int tl = 0;   // last local row that starts before the end of the tile chunk being recycled
@@ -366,9 +371,16 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   } else {
     // ===================== epilogue warps: group g drains the accumulators of MMA warps 2g, 2g+1
     const int ew = warp - kMmaWarps;
+    if constexpr (!is_partial(kEpi)) {   // bias slice of this CTA's rows (16-bit pairs)
+      pdl_wait();
+      const uint32_t* bsrc = static_cast<const uint32_t*>(sg.bias);
+      for (int i = ew * 32 + lane; i < nrows * 8; i += kEpiWarps * 32)
+        bar.bias_s[i] = bsrc ? __ldg(bsrc + (size_t)pc.i0 * 8 + i) : 0u;
+      named_bar_sync(1, kEpiWarps * 32);
+    }
     const int g = ew >> 2;
     const int quarter = warp & 3;               // TMEM lane quarter this warp may access
-    uint8_t* st = sStage + ew * 4096;
+    uint8_t* st = sStage + ew * SM::kStageWarp;
     // Per round: wait for the group's 2 accumulators (rows 8k + 2g + a), read their 32 columns with
     // one TMEM load, release them to the MMA warps, THEN do the bias / activation / store math (so
     // an MMA warp never waits for another row's epilogue arithmetic).
@@ -514,10 +526,10 @@ et_status launch_typed(const CUtensorMap& tm, const CUtensorMap& tmy, const Para
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [&] {
-    attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+    attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Smem<kEpi>::kBytes);
   });
   ET_CUDA(attr_err);
-  ET_CUDA(launch_pdl(kern, grid, dim3(kThreads), kSmemBytes, stream, tm, tmy, prm));
+  ET_CUDA(launch_pdl(kern, grid, dim3(kThreads), Smem<kEpi>::kBytes, stream, tm, tmy, prm));
   count_launch();
   return ET_OK;
 }
