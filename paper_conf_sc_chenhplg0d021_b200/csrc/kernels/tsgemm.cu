@@ -52,8 +52,19 @@ __device__ __forceinline__ unsigned long long gtime() {
   do {                                                                           \
     if (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0 && (slot) < 512) g_timeline[(slot)] = gtime(); \
   } while (0)
+// earliest stamp wins (slots 400..511 are reset to all-ones at kernel start)
+#define ET_TL_MIN(slot)                                                          \
+  do {                                                                           \
+    if (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0) atomicMin(&g_timeline[(slot)], gtime()); \
+  } while (0)
+#define ET_TL_RESET()                                                            \
+  do {                                                                           \
+    if (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0 && threadIdx.x < 112) g_timeline[400 + threadIdx.x] = ~0ull; \
+  } while (0)
 #else
 #define ET_TL(slot) do {} while (0)
+#define ET_TL_MIN(slot) do {} while (0)
+#define ET_TL_RESET() do {} while (0)
 #endif
 
 namespace {
@@ -188,11 +199,17 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
 
   if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
-  // A chunks are loaded in a rotated order: the CTAs of one token block (its pieces) start a quarter
-  // of the block apart, so they do not all hit the same L2 lines at the same moment.
+  // A chunks are loaded in K order (the first round's MMAs follow the fill chunk by chunk).
+  // ET_GEMM_A_ROT: rotate the order per piece instead (CTAs of one token block start a quarter of
+  // the block apart) — measured no faster: the L2 serves the sharing CTAs well (profiles/r01).
+#ifdef ET_GEMM_A_ROT
   const int a_rot = (blockIdx.x & 3) * (nk >> 2);
+#else
+  constexpr int a_rot = 0;
+#endif
   auto a_chunk = [&](int sq) { return sq + a_rot < nk ? sq + a_rot : sq + a_rot - nk; };
   if (threadIdx.x == 0) ET_TL(0);
+  ET_TL_RESET();
   if (threadIdx.x == 0) {
     for (int i = 0; i < kMaxKChunks; ++i) {
       mbar_init(&bar.xfull[i], 1);
@@ -315,27 +332,26 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       // one chunk: wait for the chunk once, read the tile columns lane-parallel, issue the MMAs from
       // register broadcasts.  The first segment is prepared BEFORE waiting for the accumulator, so
       // the barrier / shared-memory / shuffle latency stays off the accumulator's critical path.
-      int qb = q0, qe = q0, n = 0;
+      int qb = q0, qe = q0, n = 0, mycol = 0;
+      bool a_wait = false;
       uint32_t acol = 0, blo = 0, bhi = 0;
       auto prep = [&]() {
         const int c = qb / kChunkTiles;
         qe = min(q1, (c + 1) * kChunkTiles);
         if (c != cur_chunk) {
           mbar_wait_warp(&bar.bfull[c], 0);
+          if (lane == 0 && c < 40) ET_TL_MIN(400 + c);   // first time any MMA warp saw tile chunk c (debug)
           cur_chunk = c;
           tc_fence_after();
         }
         const int slot = (nk + c) % kSlots;
         const int coff = (pb + c * kChunkTiles) & 3;
         n = qe - qb;
-        const int mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
-        int maxcol = mycol;
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) maxcol = max(maxcol, __shfl_xor_sync(0xffffffffu, maxcol, o));
-        if ((maxcol >> 2) > a_ready) {   // every A chunk up to the segment's last tile column
-          while (a_ready < (maxcol >> 2)) mbar_wait_warp(&bar.afill[++a_ready], 0);
-          tc_fence_after();
-        }
+        mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
+        // tile columns ascend within a row: the segment's last tile has its largest column.  If an
+        // A chunk it needs is not in TMEM yet (first round: the fill is still streaming in), the
+        // issue loop waits per MMA group, so the first MMAs overlap the rest of the fill.
+        a_wait = (__shfl_sync(0xffffffffu, mycol, n - 1) >> 2) > a_ready;
         // B descriptor of tile u: start address field advances by 512 B / 16 = 32 per tile
         const uint64_t bd0 = make_sdesc(ring_u32 + slot * kSlotBytes + (qb % kChunkTiles) * 512, 128, 256,
                                         kLayoutNone);
@@ -351,7 +367,18 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k);
       while (qb < q1) {
         int u = 0;
+        auto need_a = [&](int last) {   // A chunks up to tile `last`'s column must be in TMEM
+          const int ch = __shfl_sync(0xffffffffu, mycol, last) >> 2;
+          if (ch > a_ready) {
+            while (a_ready < ch) {
+              mbar_wait_warp(&bar.afill[++a_ready], 0);
+              if (lane == 0 && warp == 0) ET_TL(450 + a_ready);
+            }
+            tc_fence_after();
+          }
+        };
         for (; u + 4 <= n; u += 4) {
+          if (a_wait) need_a(u + 3);
           if (lane == 0 && k < 8 && qb + u == q0) ET_TL(16 + 24 * warp + 3 * k + 1);
           mma_ts_warp_x4(d_tmem, __shfl_sync(0xffffffffu, acol, u), __shfl_sync(0xffffffffu, acol, u + 1),
                          __shfl_sync(0xffffffffu, acol, u + 2), __shfl_sync(0xffffffffu, acol, u + 3),
@@ -359,6 +386,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
                          (qb + u) != q0);
         }
         for (; u < n; ++u) {
+          if (a_wait) need_a(u);
           const uint32_t a = __shfl_sync(0xffffffffu, acol, u);
           mma_ts_warp_nc(d_tmem, a, ((uint64_t)bhi << 32) | (blo + 32 * u), idesc, (qb + u) != q0);
         }

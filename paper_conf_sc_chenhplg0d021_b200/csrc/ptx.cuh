@@ -43,14 +43,20 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
                : "memory");
 }
+// try_wait suspends the waiting thread (up to this many ns) until the phase completes instead of
+// returning at once: spinning waiters would otherwise take issue slots from the MMA / epilogue warps
+// sharing their SM sub-partition.
+#ifndef ET_MBAR_SUSPEND_NS
+#define ET_MBAR_SUSPEND_NS 0x989680
+#endif
 __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
   uint32_t ok;
   asm volatile(
       "{\n .reg .pred p;\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n"
       " selp.u32 %0, 1, 0, p;\n}\n"
       : "=r"(ok)
-      : "r"(smem_u32(bar)), "r"(parity)
+      : "r"(smem_u32(bar)), "r"(parity), "r"(ET_MBAR_SUSPEND_NS)
       : "memory");
   return ok != 0;
 }

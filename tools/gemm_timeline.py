@@ -22,8 +22,11 @@ for name, w, x, epi, b in [("wq", "wq", X, et.EPI_BIAS_SCALE, "bq"), ("ffn1", "w
     t = np.array(buf, dtype=np.int64)
     t0 = t[0]
     rel = lambda i: int(t[i] - t0) if t[i] >= t0 and t[i] - t0 < 10**7 else -1
+    t[t == np.iinfo(np.int64).min] = -1
     print(f"== {name}: end {rel(500)} cyc, staged {rel(1)}, A chunks " + " ".join(str(rel(2 + j)) for j in range(12))
           + f" | tiles issued {rel(14)}")
+    print("  tile chunk first seen: " + " ".join(str(rel(400 + c)) for c in range(12)) +
+          " | A chunk seen by w0: " + " ".join(str(rel(450 + j)) for j in range(12)))
     for w in range(8):
         print(f"  mma w{w}: " + " ".join(f"[{rel(16+24*w+3*k)},{rel(17+24*w+3*k)},{rel(18+24*w+3*k)}]" for k in range(6)))
     for g in range(4):
