@@ -3,6 +3,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <utility>
+#include <cstdlib>
 #include <cstdarg>
 #include <cstdint>
 #include <cstddef>
@@ -111,6 +112,9 @@ struct AttnArgs {
   unsigned long long* ts;   // trace slot or nullptr
 };
 et_status attention_run(const AttnArgs& a, cudaStream_t stream);
+// seq_len <= 128, d_k = 64, dense V: the 3-CTAs-per-SM kernel (kernels/attention128.cu)
+bool attention128_applies(const AttnArgs& a);
+et_status attention128_run(const AttnArgs& a, cudaStream_t stream);
 int attn_short_max(int d_k);
 
 // ---------------------------------------------------------------- small helpers (kernels/layernorm.cu)
@@ -134,6 +138,12 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream);
 // ---------------------------------------------------------------- tracing (api.cu)
 // Record a mark of `kind` on `stream` if tracing is enabled; counts one kernel launch.
 unsigned long long* trace_slot(int kind);
+
+// Diagnostic switches read from the environment (e.g. ET_ATTN_GENERIC=1: skip specialised kernels).
+inline bool getenv_flag(const char* name) {
+  const char* v = std::getenv(name);
+  return v != nullptr && v[0] != 0 && v[0] != '0';
+}
 
 // Launch with programmatic stream serialisation (PDL): the kernel may begin while the previous
 // kernel on the stream finishes; it must call pdl_wait() (ptx.cuh) before touching global data.

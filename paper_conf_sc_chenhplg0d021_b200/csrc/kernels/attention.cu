@@ -503,6 +503,7 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   if (!a.long_form && a.seq_len > 256) return fail(ET_ERR_UNSUPPORTED, "attention: short form needs seq_len <= 256");
   if (a.batch <= 0 || a.seq_len <= 0 || a.head_end <= a.head_begin) return ET_OK;
   if (!aligned16(a.qkv) || (a.ld_qkv * 2) % 16) return fail(ET_ERR_INVALID_ARG, "attention: QKV not 16B aligned");
+  if (attention128_applies(a) && !getenv_flag("ET_ATTN_GENERIC")) return attention128_run(a, stream);
   const uint64_t rows = (uint64_t)a.batch * a.seq_len;
   const uint32_t box_rows = rows < 128 ? (uint32_t)rows : 128u;
   CUtensorMap tm, tz;
