@@ -99,9 +99,12 @@ struct SegDev {
   float scale;
   int apply_scale;
 };
+// A piece = the tile rows one CTA computes: rows [i0, i1) of segment `seg` (seg1 == seg), or - when
+// it spans two output-contiguous segments (seg1 == seg + 1, e.g. the Q|K|V projection) - rows
+// [i0, rows(seg)) of `seg` followed by rows [0, i1) of `seg1` ("part A" and "part B").
 struct Piece {
-  int16_t seg;
-  int16_t i0, i1;  // tile rows [i0, i1) of the segment
+  int16_t seg, seg1;
+  int16_t i0, i1;
 };
 struct Params {
   int M, K, Kp, kparts;   // Kp = 768 (K part width); the last part may be shorter
@@ -131,6 +134,8 @@ struct __align__(16) Barriers {
   uint32_t bias_s[kMaxRows * 8]; // this CTA's bias slice (16-bit pairs)
   uint32_t tmem_base;
   int rows_seen[kEpiGroups];     // per epilogue group: rows whose MMAs were observed complete (in order)
+  int tcoff[kMaxSlots];          // per slot: offset of the chunk's first column index in tcol[slot]
+  int a_end;                     // end (relative tile index) of part A's last row
 };
 
 // Per epilogue: staging per epilogue warp (32 rows x 32 columns: 128 B rows in FP32, 64 B in 16-bit)
@@ -188,14 +193,20 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const Piece pc = p.piece[blockIdx.x];
-  const SegDev& sg = p.seg[pc.seg];
+  const bool two = pc.seg1 != pc.seg;
+  const SegDev& sa = p.seg[pc.seg];
+  const SegDev& sb = p.seg[pc.seg1];
   const int m0 = blockIdx.y * 128;
   const int z = blockIdx.z;
   const int nk = min(p.Kp, p.K - z * p.Kp) / 64;   // A chunks (64 K each) of this K part
-  const int32_t* rp = sg.prp + (size_t)z * (sg.tile_rows + 1);
-  const int pb = rp[pc.i0], pe = rp[pc.i1];    // this CTA's packed tiles [pb, pe)
-  const int nchunks = (pe - pb + kChunkTiles - 1) / kChunkTiles;
-  const int nrows = pc.i1 - pc.i0;
+  const int rowsA = (two ? sa.tile_rows : pc.i1) - pc.i0, rowsB = two ? pc.i1 : 0;
+  const int32_t* rpa = sa.prp + (size_t)z * (sa.tile_rows + 1);
+  const int32_t* rpb = sb.prp + (size_t)z * (sb.tile_rows + 1);
+  const int pbA = rpa[pc.i0], peA = rpa[pc.i0 + rowsA];     // part A's packed tiles [pbA, peA)
+  const int pbB = two ? rpb[0] : 0, peB = two ? rpb[rowsB] : 0;
+  const int nchA = (peA - pbA + kChunkTiles - 1) / kChunkTiles;   // part B starts on a fresh tile chunk
+  const int nchunks = nchA + (peB - pbB + kChunkTiles - 1) / kChunkTiles;
+  const int nrows = rowsA + rowsB;
   const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
 
   if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
@@ -229,13 +240,18 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   // this overlaps the previous kernel's tail under PDL).  Everything the predecessor produces (A,
   // and a bias it may have computed) is read only after pdl_wait(): by the producer before its
   // first load and by the epilogue warps before they stage the bias.
-  for (int i = threadIdx.x; i <= nrows; i += blockDim.x) bar.rptr[i] = rp[pc.i0 + i] - pb;
+  for (int i = threadIdx.x; i <= nrows; i += blockDim.x)
+    bar.rptr[i] = i < rowsA ? rpa[pc.i0 + i] - pbA
+                            : (two ? nchA * kChunkTiles + rpb[i - rowsA] - pbB : peA - pbA);
+  if (threadIdx.x == 0) bar.a_end = two ? peA - pbA : 0x7fffffff;
   pdl_trigger();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = bar.tmem_base;
   if (threadIdx.x == 0) ET_TL(1);
+  // end of local row t's tiles (part A's last row ends before the padding to part B's first chunk)
+  auto rend = [&](int t) { return t == rowsA - 1 ? min(bar.a_end, bar.rptr[t + 1]) : bar.rptr[t + 1]; };
 
   if (warp < kWarpP) {
     // A fill, smem ring -> TMEM through registers: chunk j is moved by the four warps of set j % 6,
@@ -278,7 +294,6 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       pdl_wait();
       if (p.ts != nullptr) atomicMin(p.ts, globaltimer_ns());   // trace: this CTA's work starts
       const int kx0 = z * p.Kp;
-      const uint8_t* vals = sg.values + (size_t)pb * 512;
       int tl = 0;   // last local row that starts before the end of the tile chunk being recycled
       const int nseq = nk + nchunks;
       for (int s = 0; s < nseq; ++s) {
@@ -304,14 +319,18 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           tma_load_2d(dst, &tmap_x, &bar.xfull[s], kx0 + a_chunk(s) * 64, m0);
         } else {
           const int c = s - nk;
-          const int nt = min(kChunkTiles, pe - pb - c * kChunkTiles);
+          const bool inB = c >= nchA;
+          const SegDev& sx = inB ? sb : sa;
+          const int cc = inB ? c - nchA : c, pbx = inB ? pbB : pbA, pex = inB ? peB : peA;
+          const int nt = min(kChunkTiles, pex - pbx - cc * kChunkTiles);
           // tile columns: copy from the 16-byte aligned start at or below the chunk's first entry
           // (tile_col is allocated with 16 bytes of slack, et_prune_pack_query)
-          const int first = pb + c * kChunkTiles, off = first & 3;
+          const int first = pbx + cc * kChunkTiles, off = first & 3;
           const int col_bytes = ((off + nt) * 4 + 15) & ~15;
+          bar.tcoff[slot] = off;   // published by the expect_tx arrive (release) below
           mbar_expect_tx(&bar.bfull[c], nt * 512 + col_bytes);
-          bulk_load(dst, vals + (size_t)c * kChunkTiles * 512, nt * 512, &bar.bfull[c]);
-          bulk_load(&bar.tcol[slot][0], sg.tile_col + (first - off), col_bytes, &bar.bfull[c]);
+          bulk_load(dst, sx.values + (size_t)first * 512, nt * 512, &bar.bfull[c]);
+          bulk_load(&bar.tcol[slot][0], sx.tile_col + (first - off), col_bytes, &bar.bfull[c]);
         }
       }
       ET_TL(14);
@@ -327,7 +346,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     for (int k = 0; k < nrounds; ++k) {
       const int t = k * kMmaWarps + warp;
       if (t >= nrows) break;
-      const int q0 = bar.rptr[t], q1 = bar.rptr[t + 1];   // this row's tiles, relative to pb
+      const int q0 = bar.rptr[t], q1 = rend(t);   // this row's tiles, relative to the CTA's stream
       // The row's tiles lie in chunks [q0 / 32, (q1 - 1) / 32].  A segment = the row's tiles inside
       // one chunk: wait for the chunk once, read the tile columns lane-parallel, issue the MMAs from
       // register broadcasts.  The first segment is prepared BEFORE waiting for the accumulator, so
@@ -345,7 +364,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           tc_fence_after();
         }
         const int slot = (nk + c) % kSlots;
-        const int coff = (pb + c * kChunkTiles) & 3;
+        const int coff = two ? bar.tcoff[slot] : (pbA + c * kChunkTiles) & 3;
         n = qe - qb;
         mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
         // tile columns ascend within a row: the segment's last tile has its largest column.  If an
@@ -401,9 +420,12 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     const int ew = warp - kMmaWarps;
     if constexpr (!is_partial(kEpi)) {   // bias slice of this CTA's rows (16-bit pairs)
       pdl_wait();
-      const uint32_t* bsrc = static_cast<const uint32_t*>(sg.bias);
-      for (int i = ew * 32 + lane; i < nrows * 8; i += kEpiWarps * 32)
-        bar.bias_s[i] = bsrc ? __ldg(bsrc + (size_t)pc.i0 * 8 + i) : 0u;
+      for (int i = ew * 32 + lane; i < nrows * 8; i += kEpiWarps * 32) {
+        const int t = i >> 3;
+        const uint32_t* bsrc = static_cast<const uint32_t*>(t < rowsA ? sa.bias : sb.bias);
+        const int row = t < rowsA ? pc.i0 + t : t - rowsA;
+        bar.bias_s[i] = bsrc ? __ldg(bsrc + (size_t)row * 8 + (i & 7)) : 0u;
+      }
       named_bar_sync(1, kEpiWarps * 32);
     }
     const int g = ew >> 2;
@@ -434,7 +456,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
 #pragma unroll
       for (int a = 0; a < 2; ++a) {
         const int t = t0 + min(a, na - 1);
-        const bool empty_row = a >= na || bar.rptr[t + 1] == bar.rptr[t];
+        const bool empty_row = a >= na || rend(t) == bar.rptr[t];
 #pragma unroll
         for (int c = 0; c < 16; c += 2) {
           // a row with no kept tile was never written: its accumulator is zero (output = epi(bias))
@@ -444,7 +466,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
             const float2 bb = unpack2<kBF16>(bar.bias_s[t * 8 + c / 2]);
             uint64_t xx = fadd2(f2pk(x0, x1), f2pk(bb.x, bb.y));
             if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
-              if (sg.apply_scale) xx = fmul2(xx, f2pk(sg.scale, sg.scale));
+              const SegDev& st_seg = t < rowsA ? sa : sb;
+              if (st_seg.apply_scale) xx = fmul2(xx, f2pk(st_seg.scale, st_seg.scale));
             }
             const float2 xf = f2upk(xx);
             x0 = xf.x;
@@ -464,7 +487,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       // store: registers -> this warp's 32-row staging tile -> one TMA tensor store (clipped at M by
       // the tensor map).  fp32: 128-byte rows, SWIZZLE_128B (unit c of row r at c ^ (r % 8));
       // 16-bit: 64-byte rows, SWIZZLE_64B (unit c of row r at c ^ ((r / 2) % 4)); both conflict-free.
-      const int col0 = sg.out_col + (pc.i0 + t0) * 16;
+      // output columns: segments of a two-part piece are output-contiguous (checked on the host)
+      const int col0 = t0 < rowsA ? sa.out_col + (pc.i0 + t0) * 16 : sb.out_col + (t0 - rowsA) * 16;
       const int row0 = m0 + quarter * 32;
       if (na == 2) {
         if (lane == 0) bulk_wait_group_read<0>();   // the previous store finished reading the staging tile
@@ -648,7 +672,6 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   int pieces_total = target_ctas / (mblocks * kparts);
   if (pieces_total < 1) pieces_total = 1;
   if (pieces_total < a.nseg) pieces_total = a.nseg;
-  int np = 0;
   for (int s = 0; s < a.nseg; ++s) {
     const GemmSegment& gs = a.seg[s];
     prm.seg[s].prp = gs.row_ptr;
@@ -659,32 +682,71 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     prm.seg[s].out_col = gs.out_col;
     prm.seg[s].scale = gs.scale;
     prm.seg[s].apply_scale = gs.apply_scale;
-    int ps = (int)(((long long)pieces_total * gs.tile_rows * 2 + (total_rows > 0 ? total_rows : 1)) /
-                   (2LL * (total_rows > 0 ? total_rows : 1)));   // rounded
-    if (ps < 1) ps = 1;
-    if (ps > gs.tile_rows / 8) ps = gs.tile_rows / 8 > 0 ? gs.tile_rows / 8 : 1;
-    // each piece's tile stream must fit kMaxBChunks chunks
-    for (;;) {
-      bool ok = true;
+  }
+  const int kt = std::min(a.K, 768) / 16;   // tile columns per K part (bound on tiles per row)
+  auto fits = [&](int rows) { return rows <= kMaxRows && (long long)rows * kt + kChunkTiles <= (long long)kMaxBChunks * kChunkTiles; };
+  int np = 0;
+  // Output-contiguous segments (Q|K|V): plan the pieces over the concatenated tile rows, so the CTA
+  // count is set by the total rows rather than rounded per segment (4 pieces of 36 rows instead of
+  // 3 of 48 for BERT-base); a piece may straddle one segment boundary.
+  bool contiguous = a.nseg > 1;
+  for (int s = 1; s < a.nseg; ++s)
+    contiguous = contiguous && a.seg[s].out_col == a.seg[s - 1].out_col + a.seg[s - 1].tile_rows * 16;
+  if (contiguous) {
+    int start[4] = {0, 0, 0, 0};
+    for (int s = 0; s < a.nseg; ++s) start[s + 1] = start[s] + a.seg[s].tile_rows;
+    const int q4 = (total_rows + 3) / 4;
+    int ps = std::max(1, std::min(pieces_total, q4));
+    bool ok = false;
+    for (; ps <= q4 && !ok; ++ps) {
+      ok = true;
+      np = 0;
       for (int k = 0; k < ps && ok; ++k) {
-        const int q4 = (gs.tile_rows + 3) / 4;
-        const int i0 = std::min(gs.tile_rows, 4 * (int)((long long)q4 * k / ps));
-        const int i1 = std::min(gs.tile_rows, 4 * (int)((long long)q4 * (k + 1) / ps));
-        ok = (long long)(i1 - i0) * (std::min(a.K, 768) / 16) <= (long long)kMaxBChunks * kChunkTiles &&
-             i1 - i0 <= kMaxRows;
+        const int g0 = std::min(total_rows, 4 * (int)((long long)q4 * k / ps));
+        const int g1 = std::min(total_rows, 4 * (int)((long long)q4 * (k + 1) / ps));
+        if (g1 <= g0) continue;
+        int s0 = 0;
+        while (g0 >= start[s0 + 1]) ++s0;
+        int s1 = s0;
+        while (g1 > start[s1 + 1]) ++s1;
+        if (s1 > s0 + 1 || !fits(g1 - g0) || np >= kMaxPieces) {
+          ok = false;
+          break;
+        }
+        prm.piece[np].seg = (int16_t)s0;
+        prm.piece[np].seg1 = (int16_t)s1;
+        prm.piece[np].i0 = (int16_t)(g0 - start[s0]);
+        prm.piece[np].i1 = (int16_t)(g1 - start[s1]);
+        ++np;
       }
-      if (ok || ps >= (gs.tile_rows + 3) / 4) break;
-      ++ps;
     }
-    ps = std::min(ps, (gs.tile_rows + 3) / 4);   // no empty pieces
-    for (int k = 0; k < ps; ++k) {
-      if (np >= kMaxPieces) return fail(ET_ERR_INTERNAL, "tile GEMM: too many pieces");
-      prm.piece[np].seg = (int16_t)s;
-      // piece boundaries on multiples of 4 tile rows (an epilogue quad never straddles two CTAs)
+    if (!ok) contiguous = false;
+  }
+  if (!contiguous) {
+    np = 0;
+    for (int s = 0; s < a.nseg; ++s) {
+      const GemmSegment& gs = a.seg[s];
+      int ps = (int)(((long long)pieces_total * gs.tile_rows * 2 + (total_rows > 0 ? total_rows : 1)) /
+                     (2LL * (total_rows > 0 ? total_rows : 1)));   // rounded
+      ps = std::max(1, std::min(ps, std::max(1, gs.tile_rows / 8)));
       const int q4 = (gs.tile_rows + 3) / 4;
-      prm.piece[np].i0 = (int16_t)std::min(gs.tile_rows, 4 * (int)((long long)q4 * k / ps));
-      prm.piece[np].i1 = (int16_t)std::min(gs.tile_rows, 4 * (int)((long long)q4 * (k + 1) / ps));
-      ++np;
+      for (;;) {   // each piece's tile stream must fit the per-CTA chunk / row budgets
+        bool ok = true;
+        for (int k = 0; k < ps && ok; ++k)
+          ok = fits(std::min(gs.tile_rows, 4 * (int)((long long)q4 * (k + 1) / ps)) -
+                    std::min(gs.tile_rows, 4 * (int)((long long)q4 * k / ps)));
+        if (ok || ps >= q4) break;
+        ++ps;
+      }
+      ps = std::min(ps, q4);   // no empty pieces
+      for (int k = 0; k < ps; ++k) {
+        if (np >= kMaxPieces) return fail(ET_ERR_INTERNAL, "tile GEMM: too many pieces");
+        prm.piece[np].seg = prm.piece[np].seg1 = (int16_t)s;
+        // piece boundaries on multiples of 4 tile rows (an epilogue pair never straddles two CTAs)
+        prm.piece[np].i0 = (int16_t)std::min(gs.tile_rows, 4 * (int)((long long)q4 * k / ps));
+        prm.piece[np].i1 = (int16_t)std::min(gs.tile_rows, 4 * (int)((long long)q4 * (k + 1) / ps));
+        ++np;
+      }
     }
   }
   prm.npieces = np;
