@@ -43,6 +43,8 @@ namespace et {
 //   round k: accumulator free / first MMA / commit; 208 + 40*g + 5*k + {0,1,2,3}: epilogue group g,
 //   round k: pair complete / drained / math done / stores issued; 500: end.
 __device__ unsigned long long g_timeline[512];
+// per-CTA (start, end) %globaltimer and SM id of the most recent launch (debug builds)
+__device__ unsigned long long g_cta_span[2048][3];
 __device__ __forceinline__ unsigned long long gtime() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
@@ -126,7 +128,7 @@ struct __align__(16) Barriers {
   // parity wait on a reused barrier cannot tell those phases apart)
   uint64_t xfull[kMaxKChunks];   // A load #s landed in its slot (TMA transaction bytes)
   uint64_t xfree[kMaxKChunks];   // A load #s read out of its slot (4 fill warps)
-  uint64_t afill[kMaxKChunks];   // A chunk j stored into TMEM (4 fill warps)
+  uint64_t a_all;                // the whole A block is in TMEM (4 fill warps x nk chunks)
   uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
   uint64_t bfull[kMaxBChunks];
   alignas(16) int tcol[kMaxSlots][kChunkTiles + 4];   // bulk-copy destination (16-byte aligned): tile columns
@@ -221,12 +223,21 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   auto a_chunk = [&](int sq) { return sq + a_rot < nk ? sq + a_rot : sq + a_rot - nk; };
   if (threadIdx.x == 0) ET_TL(0);
   ET_TL_RESET();
+#ifdef ET_TIMELINE
+  const unsigned cta_lin = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+  if (threadIdx.x == 0 && cta_lin < 2048) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    g_cta_span[cta_lin][0] = globaltimer_ns();
+    g_cta_span[cta_lin][2] = smid;
+  }
+#endif
   if (threadIdx.x == 0) {
     for (int i = 0; i < kMaxKChunks; ++i) {
       mbar_init(&bar.xfull[i], 1);
       mbar_init(&bar.xfree[i], 4);
-      mbar_init(&bar.afill[i], 4);
     }
+    mbar_init(&bar.a_all, 4 * nk);
     for (int i = 0; i < kMmaWarps; ++i) {
       mbar_init(&bar.acc_full[i], 1);
       mbar_init(&bar.acc_empty[i], 4);
@@ -278,7 +289,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       tmem_st_wait();
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&bar.afill[j]);
+      if (lane == 0) mbar_arrive(&bar.a_all);
       if (lane == 0 && q == 0) ET_TL(2 + sq);
     }
   }
@@ -341,8 +352,11 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     const uint32_t d_tmem = tbase + kAccCol + warp * 16;
     const uint32_t ring_u32 = smem_u32(ring);
     const int kbase = z * 48;   // first tile column of this K part
-    int a_ready = -1;           // highest A chunk known filled
     int cur_chunk = -1;         // tile chunk whose full barrier was last waited
+    // one wait for the whole A block (a wait on a completed mbarrier still costs ~100-300 cycles
+    // of this warp's issue: per-chunk waits made the first round 2-3x slower than the others)
+    mbar_wait_warp(&bar.a_all, 0);
+    tc_fence_after();
     for (int k = 0; k < nrounds; ++k) {
       const int t = k * kMmaWarps + warp;
       if (t >= nrows) break;
@@ -352,7 +366,6 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       // register broadcasts.  The first segment is prepared BEFORE waiting for the accumulator, so
       // the barrier / shared-memory / shuffle latency stays off the accumulator's critical path.
       int qb = q0, qe = q0, n = 0, mycol = 0;
-      bool a_wait = false;
       uint32_t acol = 0, blo = 0, bhi = 0;
       auto prep = [&]() {
         const int c = qb / kChunkTiles;
@@ -367,10 +380,6 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         const int coff = two ? bar.tcoff[slot] : (pbA + c * kChunkTiles) & 3;
         n = qe - qb;
         mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
-        // tile columns ascend within a row: the segment's last tile has its largest column.  If an
-        // A chunk it needs is not in TMEM yet (first round: the fill is still streaming in), the
-        // issue loop waits per MMA group, so the first MMAs overlap the rest of the fill.
-        a_wait = (__shfl_sync(0xffffffffu, mycol, n - 1) >> 2) > a_ready;
         // B descriptor of tile u: start address field advances by 512 B / 16 = 32 per tile
         const uint64_t bd0 = make_sdesc(ring_u32 + slot * kSlotBytes + (qb % kChunkTiles) * 512, 128, 256,
                                         kLayoutNone);
@@ -386,18 +395,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k);
       while (qb < q1) {
         int u = 0;
-        auto need_a = [&](int last) {   // A chunks up to tile `last`'s column must be in TMEM
-          const int ch = __shfl_sync(0xffffffffu, mycol, last) >> 2;
-          if (ch > a_ready) {
-            while (a_ready < ch) {
-              mbar_wait_warp(&bar.afill[++a_ready], 0);
-              if (lane == 0 && warp == 0) ET_TL(450 + a_ready);
-            }
-            tc_fence_after();
-          }
-        };
         for (; u + 4 <= n; u += 4) {
-          if (a_wait) need_a(u + 3);
           if (lane == 0 && k < 8 && qb + u == q0) ET_TL(16 + 24 * warp + 3 * k + 1);
           mma_ts_warp_x4(d_tmem, __shfl_sync(0xffffffffu, acol, u), __shfl_sync(0xffffffffu, acol, u + 1),
                          __shfl_sync(0xffffffffu, acol, u + 2), __shfl_sync(0xffffffffu, acol, u + 3),
@@ -405,7 +403,6 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
                          (qb + u) != q0);
         }
         for (; u < n; ++u) {
-          if (a_wait) need_a(u);
           const uint32_t a = __shfl_sync(0xffffffffu, acol, u);
           mma_ts_warp_nc(d_tmem, a, ((uint64_t)bhi << 32) | (blo + 32 * u), idesc, (qb + u) != q0);
         }
@@ -545,6 +542,9 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   tc_fence_before();
   __syncthreads();
   if (threadIdx.x == 0) ET_TL(500);
+#ifdef ET_TIMELINE
+  if (threadIdx.x == 0 && cta_lin < 2048) g_cta_span[cta_lin][1] = globaltimer_ns();
+#endif
   trace_cta_end(p.ts);
   if (warp == kWarpP) {
     __syncwarp();
@@ -783,6 +783,9 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
 }
 
 #ifdef ET_TIMELINE
+extern "C" int et_diag_gemm_cta_spans(unsigned long long* host_out) {
+  return cudaMemcpyFromSymbol(host_out, g_cta_span, sizeof(g_cta_span)) == cudaSuccess ? 0 : 4;
+}
 extern "C" int et_diag_gemm_timeline(unsigned long long* host_out) {
   return cudaMemcpyFromSymbol(host_out, g_timeline, sizeof(g_timeline)) == cudaSuccess ? 0 : 4;
 }

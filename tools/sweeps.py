@@ -1,0 +1,84 @@
+"""SURVEY §8(d) diagnostics beside the headline (run on the GPU box; JSON lines to stdout):
+  M2  sparsity sweep (Fig. 10 / line 252 analogue): the tile-sparse linear layer at M = 4096
+      tokens for d x d (d = 768, 1024) and the BERT FFN shapes, tile ratio 0 ... 0.95;
+  M3  sequence-length crossover (Fig. 8 / line 244 analogue): short vs long attention form at fixed
+      total tokens, BERT-base heads (H = 12, d_k = 64).
+Timing: CUDA events around 50 back-to-back launches after 5 warm-ups (operands L2-resident when they
+fit: a kernel-level diagnostic, not the bench metric).  Dense torch.matmul at the same shape is
+printed as context only (it is never a backend)."""
+import json, math, os, sys
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_sc_chenhplg0d021_b200 as et  # noqa: E402
+from et_synth import make_matrix  # noqa: E402
+
+PEAK = {"hbm_gbs": 6547.5, "tc_tflops": 1642.5}
+try:
+    PEAK.update({k: v for k, v in json.load(open("MEASURED_PEAKS.json")).items() if k in ("hbm_gbs",)})
+    PEAK["tc_tflops"] = json.load(open("MEASURED_PEAKS.json")).get("bf16_tflops", PEAK["tc_tflops"])
+except Exception:
+    pass
+
+
+def timed(fn, reps=50, warm=5):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(True), torch.cuda.Event(True)
+    a.record()
+    for _ in range(reps):
+        fn()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / reps * 1e3   # us
+
+
+def m2():
+    M = 4096
+    shapes = [("d768", 768, 768), ("d1024", 1024, 1024), ("ffn1", 3072, 768), ("ffn2", 768, 3072)]
+    for name, N, K in shapes:
+        W = torch.tensor(make_matrix(5, (N, K), 0.02, "fp16"), dtype=torch.float16, device="cuda")
+        X = torch.tensor(make_matrix(6, (M, K), 1.0, "fp16"), dtype=torch.float16, device="cuda")
+        dense_us = timed(lambda: torch.matmul(X, W.t()))
+        for ratio in (0.0, 0.2, 0.4, 0.6, 0.8, 0.9, 0.95):
+            pk = et.prune_pack(W, "tile", ratio)
+            nnz = pk.c.ntiles
+            epi = et.EPI_PART16 if K > 768 else et.EPI_BIAS
+            out = et.linear_fwd(pk, X, None, epi)
+            us = timed(lambda: et.linear_fwd(pk, X, None, epi, out=out))
+            flops = 2.0 * M * 256 * nnz
+            planes = (K + 767) // 768
+            nbytes = M * K * 2 + nnz * 512 + M * N * 2 * planes
+            print(json.dumps({"sweep": "M2", "shape": name, "M": M, "N": N, "K": K, "ratio": ratio, "kept_tiles": nnz,
+                              "us": round(us, 2), "eff_tflops": round(flops / us / 1e6, 1),
+                              "alg_gbs": round(nbytes / us / 1e3, 1),
+                              "hbm_roofline_frac": round(nbytes / us / 1e3 / PEAK["hbm_gbs"], 3),
+                              "dense_torch_matmul_us": round(dense_us, 2)}), flush=True)
+
+
+def m3():
+    H, dk, total = 12, 64, 32768
+    d = H * dk
+    for S in (64, 128, 192, 224, 256, 320, 384, 512, 1024, 2048):
+        B = max(1, total // S)
+        qkv = torch.randn(B * S, 3 * d, device="cuda").half()
+        Z = torch.empty(B * S, d, device="cuda").half()
+        flops = 4.0 * B * H * S * S * dk
+        row = {"sweep": "M3", "S": S, "B": B, "H": H, "d_k": dk}
+        for mode in ("short", "long"):
+            if mode == "short" and S > et.attn_short_max(dk):
+                continue
+            us = timed(lambda: et.attn_core_fwd(qkv, B, S, H, d, 0, d, 2 * d, mode=mode, scale=0.125, Z=Z))
+            row[f"{mode}_us"] = round(us, 2)
+            row[f"{mode}_eff_tflops"] = round(flops / us / 1e6, 1)
+        print(json.dumps(row), flush=True)
+
+
+if __name__ == "__main__":
+    which = sys.argv[1:] or ["m2", "m3"]
+    if "m2" in which:
+        m2()
+    if "m3" in which:
+        m3()
