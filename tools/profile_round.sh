@@ -8,7 +8,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none -c 2500 --csv --log-fi
 # 84 kernel launches per encoder call (12 layers x 7); the second call's layer-0 kernels
 ncu --set full --clock-control none --import-source on -k regex:tsgemm -s 48 -c 4 -f -o gpurun_out/prof_gemm \
     python tools/prof_layer.py > gpurun_out/prof_gemm.log 2>&1
-ncu --set full --clock-control none --import-source on -k regex:attn_kernel -s 12 -c 1 -f -o gpurun_out/prof_attn \
+ncu --set full --clock-control none --import-source on -k regex:attn -s 12 -c 1 -f -o gpurun_out/prof_attn \
     python tools/prof_layer.py > gpurun_out/prof_attn.log 2>&1
 ncu --set full --clock-control none --import-source on -k regex:layernorm -s 24 -c 2 -f -o gpurun_out/prof_ln \
     python tools/prof_layer.py > gpurun_out/prof_ln.log 2>&1
