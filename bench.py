@@ -51,6 +51,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the cpu_baseline sample")
+    ap.add_argument("--parallel", choices=["batch", "head"], default="batch",
+                    help="batch: batch sharding (default, weak scaling); head: head-parallel latency mode "
+                         "(Eq. 4 partials + NCCL all-reduce per layer, strong scaling)")
     return ap.parse_args()
 
 
@@ -476,6 +479,80 @@ def our_arm(args):
         dist.destroy_process_group()
 
 
+# ------------------------------------------------------------------------------------------ head-parallel arm
+def head_parallel_arm(args):
+    """Head-parallel latency mode: every rank runs the whole batch on its heads
+    (dist.HeadParallelEncoder), an NCCL all-reduce of the FP32 O-projection partials per layer, the
+    FFN replicated.  Total work fixed as N grows ("strong").  Eager launches (the all-reduce sits
+    between library calls), so this mode is host-launch bound at small batches."""
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py: no CUDA device (this benchmark has no CPU fallback)")
+    torch.cuda.set_device(local)
+    import torch.distributed as dist
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29518")
+    if not dist.is_initialized():
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local))
+    import paper_conf_sc_chenhplg0d021_b200 as et
+    from et_synth import CONFIGS, make_layer, make_lengths, make_x
+    from paper_conf_sc_chenhplg0d021_b200.dist import HeadParallelEncoder
+    cfg = CONFIGS[args.config]
+    dtype = cfg.dtype if cfg.dtype != "fp32" else "fp16"
+    raws = [make_layer(cfg, l) for l in range(cfg.layers)]
+    layers = [et.pack_layer(r, cfg.scheme, cfg.ratio, cfg.heads, dtype) for r in raws]
+    L = torch.from_numpy(make_lengths(cfg, ragged=False)).cuda()
+    enc = HeadParallelEncoder(raws, layers, cfg.heads, cfg.batch, cfg.seq_len, cfg.d_ff, act=cfg.act,
+                              ln_eps=cfg.ln_eps, dtype=dtype, causal=cfg.causal, mode=cfg.attn_mode, lengths=L,
+                              rank=rank, world=world, group=dist.group.WORLD)
+    X = make_x(cfg)
+    Xd = torch.from_numpy(np.ascontiguousarray(X.reshape(cfg.tokens, cfg.d_model))).cuda().to(et.torch_dtype(dtype))
+    out = torch.empty_like(Xd)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    stream = torch.cuda.current_stream()
+    for _ in range(max(args.warmup, 3)):
+        enc(Xd, out)
+    torch.cuda.synchronize()
+    K = args.steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    clk = ClockSampler(local)
+    dist.barrier()
+    torch.cuda.synchronize()
+    clk.start()
+    launches0 = et._lib.et_launch_count()
+    for s in range(K):
+        flush.fill_(float(s))
+        ev[s][0].record(stream)
+        enc(Xd, out)
+        ev[s][1].record(stream)
+    launches = et._lib.et_launch_count() - launches0
+    torch.cuda.synchronize()
+    dist.barrier()
+    clocks = clk.stop()
+    t = torch.tensor([sum(a.elapsed_time(b) for a, b in ev) / 1e3], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    t_max = float(t[0])
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": cfg.batch * K / t_max, "unit": "seqs/s", "n_gpus": world, "steps": K,
+            "warmup": max(args.warmup, 3), "ms_per_step": 1e3 * t_max / K, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": dtype, "data": "synthetic",
+            "config": {"workload": workload_name(cfg), "global_batch": cfg.batch, "seq_len": cfg.seq_len,
+                       "parallelism": f"hp{world} (head-parallel: W_O partials + NCCL all-reduce per layer, "
+                                      f"FFN replicated)",
+                       "heads_rank0": [enc.h0, enc.h1],
+                       "l2": "flushed before every timed step (256 MiB write, outside the events)",
+                       "launch": "eager (all-reduce between library calls)"},
+            "gpu_launches": int(launches), "clocks": clocks, "mode": "head-parallel (latency mode, optional)",
+        }
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
 def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -488,6 +565,9 @@ def main():
         cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
                "--master-addr", "127.0.0.1", "--master-port", "29517", __file__] + sys.argv[1:]
         raise SystemExit(subprocess.call(cmd))
+    if args.parallel == "head":
+        head_parallel_arm(args)
+        return
     our_arm(args)
 
 

@@ -165,9 +165,8 @@ et_status et_layernorm_fwd(const void* part, et_dtype part_dtype, int32_t nparts
  *                j >= len are masked (probability exactly 0, line 73; reading C-7).  NULL = all.
  *   causal       nonzero: also mask j > i (the triangular mask of line 73)
  *   mode         short / long / auto (auto: short while seq_len <= et_attn_short_max())
- *   head_begin, head_end   head range computed by this call ([0, H) normally; a sub-range in
- *                head-parallel mode, where `out` receives that range's W_O partial sum:
- *                bias only if head_begin == 0, no residual/LN — Eq. 4).
+ *   head_begin, head_end   head range computed by this call ([0, H) normally; a sub-range
+ *                [h0, h1) in head-parallel mode, see et_attention_fwd (Eq. 4).
  * ------------------------------------------------------------------------------------------ */
 typedef struct {
   int32_t batch, seq_len, heads, d_model;
@@ -199,7 +198,21 @@ et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld
  *   out = SelfAttn(X)                  if ln_gamma == NULL
  *   out = LN(X + SelfAttn(X))          otherwise (post-LN, line 75)
  * wq, wk, wo: TILE (or NONE packed as all-kept TILE); wv: TILE or ROW (attention-aware,
- * line 107/317).  Biases in dtype; ln params fp32.  X, out: [batch*seq_len, d_model] in dtype. */
+ * line 107/317).  Biases in dtype; ln params fp32.  X, out: [batch*seq_len, d_model] in dtype.
+ *
+ * Head-parallel mode (desc->head_begin/head_end = [h0, h1) != [0, H); Megatron-style split of
+ * Eq. 4: Output = sum_h Z_h . W_O,h^T, so each rank computes the sum over its heads and
+ * an all-reduce(sum) over ranks gives the full output):
+ *   wq, wk, wv  the rank's ROW slices [(h1-h0)*d_k, d_model] of the full matrices (rows h0*d_k ..),
+ *   wo          its COLUMN slice [d_model, (h1-h0)*d_k] (columns h0*d_k ..),
+ *               each packed with mask_in = the full matrix's mask restricted to the slice, so the
+ *               kept set is the one the whole-matrix ranking chose (pruning is per matrix, C-3);
+ *   bq, bk, bv  the matching slices of the biases; bo the full [d_model] bias;
+ *   ln_gamma    must be NULL (residual + LN follow the all-reduce: et_layernorm_fwd);
+ *   out         FP32 [batch*seq_len, d_model] (reading C-21: FP32 partials) =
+ *               sum_{h in [h0,h1)} Z_h W_O,h^T  + b_O (only if h0 == 0)
+ *               + sum over this rank's pruned V features f of W_O[:, f] b_V[f] (ROW W_V, C-6).
+ * Errors: ET_ERR_INVALID_ARG for slice shapes that do not match the range or a non-NULL gamma. */
 et_status et_attention_workspace_size(const et_attn_desc* desc, const et_packed_weight* wv, size_t* bytes);
 et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_packed_weight* wq,
                            const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
@@ -218,7 +231,9 @@ typedef struct {
  *   Y1 = LN(X + SelfAttn(X));  U = act(Y1 W1'^T + b1);  Y2 = LN(Y1 + U W2'^T + b2).
  * X, out: [batch*seq_len, d_model] in resid_dtype (FP32, or equal to desc->dtype; reading C-22);
  * GEMM operands in desc->dtype.  layers_host: host array of num_layers et_layer.  X and out
- * may alias.  No host synchronisation; CUDA-graph capturable. */
+ * may alias.  No host synchronisation; CUDA-graph capturable.  Full head range only
+ * (ET_ERR_UNSUPPORTED otherwise): a head-parallel layer is et_attention_fwd on the rank's slices,
+ * an all-reduce of the FP32 partials by the caller's process group, then et_layernorm_fwd. */
 et_status et_encoder_workspace_size(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff,
                                     et_dtype resid_dtype, const et_layer* layers_host, size_t* bytes);
 et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff, et_act act, float ln_eps,

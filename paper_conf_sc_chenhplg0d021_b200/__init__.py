@@ -167,7 +167,11 @@ def prune_pack(W: torch.Tensor, pattern: str = "tile", ratio: float = 0.8, tile=
     pat = _PAT[pattern] if isinstance(pattern, str) else pattern
     sizes = [_sz() for _ in range(8)]
     nnz = _i32()
-    _check(_q(rows, cols, dt, pat, ratio, tile[0], tile[1], group_rows, None, ctypes.byref(nnz),
+    # with mask_in the kept count is its popcount: the size query needs a host copy of the bitmap
+    host_mask = None
+    if mask_in is not None:
+        host_mask = mask_in.detach().to("cpu", torch.int32).contiguous()
+    _check(_q(rows, cols, dt, pat, ratio, tile[0], tile[1], group_rows, _ptr(host_mask), ctypes.byref(nnz),
               *[ctypes.byref(s) for s in sizes]))
     names = ["mask", "idx", "row_ptr", "tile_col", "row_map", "part_row_ptr", "values", "ws"]
     dev = W.device
@@ -323,22 +327,39 @@ def pack_layer(raw: dict, scheme: str, ratio: float, heads: int, dtype="fp16", s
     return Layer(packed, dense)
 
 
-def attention_fwd(X: torch.Tensor, layer: Layer, batch: int, seq_len: int, heads: int, lengths=None,
-                  causal=False, mode="auto", ln: bool = True, ln_eps: float = 1e-12, out=None, stream=None):
-    """et_attention_fwd: LN(X + SelfAttn(X)) (ln=True) or SelfAttn(X)."""
-    d_model = X.shape[1]
-    d = attn_desc(batch, seq_len, heads, d_model, X.dtype, lengths, causal, mode)
-    P, D = layer.packed, layer.dense
+def attention_workspace_size(layer: Layer, batch: int, seq_len: int, heads: int, d_model: int, dtype,
+                             head_range=None) -> int:
+    """et_attention_workspace_size (bytes)."""
+    h0, h1 = head_range or (0, heads)
+    d = attn_desc(batch, seq_len, heads, d_model, dtype, head_begin=h0, head_end=h1)
     nb = _sz()
-    _check(_attn_ws(ctypes.byref(d), ctypes.byref(P["wv"].c), ctypes.byref(nb)))
-    ws = torch.empty(nb.value, dtype=torch.uint8, device=X.device)
+    _check(_attn_ws(ctypes.byref(d), ctypes.byref(layer.packed["wv"].c), ctypes.byref(nb)))
+    return int(nb.value)
+
+
+def attention_fwd(X: torch.Tensor, layer: Layer, batch: int, seq_len: int, heads: int, lengths=None,
+                  causal=False, mode="auto", ln: bool = True, ln_eps: float = 1e-12, out=None, stream=None,
+                  head_range=None, workspace: torch.Tensor | None = None):
+    """et_attention_fwd: LN(X + SelfAttn(X)) (ln=True) or SelfAttn(X).
+
+    head_range=(h0, h1) != (0, heads): head-parallel partial (Eq. 4) — `layer` holds the rank's
+    slices (dist.pack_head_slice), no LN, out is FP32 [M, d_model]."""
+    d_model = X.shape[1]
+    h0, h1 = head_range or (0, heads)
+    hp = (h0, h1) != (0, heads)
+    d = attn_desc(batch, seq_len, heads, d_model, X.dtype, lengths, causal, mode, head_begin=h0, head_end=h1)
+    P, D = layer.packed, layer.dense
+    if workspace is None:
+        workspace = torch.empty(attention_workspace_size(layer, batch, seq_len, heads, d_model, X.dtype, (h0, h1)),
+                                dtype=torch.uint8, device=X.device)
     if out is None:
-        out = torch.empty_like(X)
+        out = torch.empty(X.shape, dtype=torch.float32 if hp else X.dtype, device=X.device)
+    use_ln = ln and not hp
     _check(_attn(ctypes.byref(d), X.data_ptr(), ctypes.byref(P["wq"].c), ctypes.byref(P["wk"].c),
                  ctypes.byref(P["wv"].c), ctypes.byref(P["wo"].c), D["bq"].data_ptr(), D["bk"].data_ptr(),
-                 D["bv"].data_ptr(), D["bo"].data_ptr(), D["ln1_g"].data_ptr() if ln else None,
-                 D["ln1_b"].data_ptr() if ln else None, ln_eps, out.data_ptr(), ws.data_ptr(), ws.numel(),
-                 _stream(stream)))
+                 D["bv"].data_ptr(), D["bo"].data_ptr(), D["ln1_g"].data_ptr() if use_ln else None,
+                 D["ln1_b"].data_ptr() if use_ln else None, ln_eps, out.data_ptr(), workspace.data_ptr(),
+                 workspace.numel(), _stream(stream)))
     return out
 
 

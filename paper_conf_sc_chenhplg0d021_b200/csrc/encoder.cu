@@ -93,16 +93,22 @@ struct BlockWs {
   void* bo_folded;  // [d]
 };
 
-int v_cols_of(const et_packed_weight* wv, int d) {
+int v_cols_of(const et_packed_weight* wv, int d) {   // d: the width W_V produces (inner width)
   return wv->pattern == ET_PRUNE_ROW ? (int)align_up((size_t)std::max(wv->rows_padded, 16), 8) : d;
 }
+
+// Inner width of the block: the Q/K/V/Z columns this call computes (d_model, or the rank's
+// (head_end - head_begin) * d_k in head-parallel mode).
+int inner_width(const et_attn_desc* d) { return (d->head_end - d->head_begin) * (d->d_model / d->heads); }
+bool head_parallel(const et_attn_desc* d) { return d->head_begin != 0 || d->head_end != d->heads; }
 
 void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, BlockWs* ws) {
   const size_t M = (size_t)d->batch * d->seq_len;
   const size_t es = dtype_size(d->dtype);
-  ws->ldq = 2 * d->d_model + vmax;
+  const int dq = inner_width(d);
+  ws->ldq = 2 * dq + vmax;
   ws->qkv = c.take(M * ws->ldq * es);
-  ws->z = c.take(M * d->d_model * es);
+  ws->z = c.take(M * dq * es);
   ws->part = c.take((size_t)kparts_max * M * d->d_model * 4);   // sized for FP32
   ws->v_col = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
   ws->v_width = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
@@ -110,24 +116,33 @@ void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, Blo
   ws->bo_folded = c.take((size_t)d->d_model * es);
 }
 
-// Steps 1-3 (+4 when gamma != NULL): attention block on X (act dtype), output either the fp32
-// O-projection partial in ws->part (for the caller's LayerNorm) or written through `ln`.
+// Steps 1-3 (+4 when gamma != NULL): attention block on X (act dtype), output the O-projection
+// partial in ws->part (for the caller's LayerNorm step, which adds *bo_eff).
+// Head-parallel mode (desc head range [h0, h1) != [0, H); Megatron-style split of Eq. 4,
+// Output = sum_h Z_h W_O,h^T): wq / wk / wv are the rank's ROW slices
+// [(h1-h0) d_k, d] of the full matrices and wo its COLUMN slice [d, (h1-h0) d_k], each packed with
+// the global mask restricted to the slice; the block computes heads h0..h1-1 only, the partial is
+// FP32 (reading C-21), and *bo_eff carries b_O only on the rank with h0 == 0 (plus this rank's
+// share of the pruned-V bias fold, reading C-6), so that the sum over ranks is the full output.
 et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et_packed_weight* wq,
                               const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
                               const void* bq, const void* bk, const void* bv, const void* bo, const BlockWs& ws,
                               const void** bo_eff, cudaStream_t st) {
-  const int dm = d->d_model, H = d->heads, dk = dm / H;
+  const int dm = d->d_model, dk = dm / d->heads;
+  const bool hp = head_parallel(d);
+  const int Hr = d->head_end - d->head_begin, dq = Hr * dk;
   const int M = d->batch * d->seq_len;
   const bool rowv = wv->pattern == ET_PRUNE_ROW;
+  const void* bo_rank = (hp && d->head_begin != 0) ? nullptr : bo;   // b_O enters the sum once
   const void* bv_use = bv;
-  *bo_eff = bo;
+  *bo_eff = bo_rank;
   if (rowv) {
-    VPrep vp{wv, wo, bv, bo, H, dk, d->dtype, ws.v_col, ws.v_width, ws.bv_packed, ws.bo_folded};
+    VPrep vp{wv, wo, bv, bo_rank, Hr, dk, d->dtype, ws.v_col, ws.v_width, ws.bv_packed, ws.bo_folded};
     ET_TRY(vprep_run(vp, st));
     bv_use = ws.bv_packed;
     *bo_eff = ws.bo_folded;
     // pruned V features leave zero columns in Z (their constant b_V is folded into b_O')
-    ET_CUDA(cudaMemsetAsync(ws.z, 0, (size_t)M * dm * dtype_size(d->dtype), st));
+    ET_CUDA(cudaMemsetAsync(ws.z, 0, (size_t)M * dq * dtype_size(d->dtype), st));
   }
   // 1. QKV projection: one launch, three segments; Q scaled by 1/sqrt(d_k) before rounding
   GemmArgs g{};
@@ -140,32 +155,32 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   g.seg[0] = seg_of(wq, bq, 0);
   g.seg[0].apply_scale = 1;
   g.seg[0].scale = 1.0f / std::sqrt((float)dk);
-  g.seg[1] = seg_of(wk, bk, dm);
-  g.seg[2] = seg_of(wv, bv_use, 2 * dm);
+  g.seg[1] = seg_of(wk, bk, dq);
+  g.seg[2] = seg_of(wv, bv_use, 2 * dq);
   g.Y = ws.qkv;
   g.ldy = ws.ldq;
   g.epi = ET_EPI_BIAS_SCALE;
   g.ts = trace_slot(ET_K_QKV);
   ET_TRY(gemm_run(g, st));
-  // 2. attention core
+  // 2. attention core over this call's heads (local indices 0..Hr-1)
   AttnArgs a{};
   a.qkv = ws.qkv;
   a.ld_qkv = ws.ldq;
   a.q_off = 0;
-  a.k_off = dm;
-  a.v_off = 2 * dm;
+  a.k_off = dq;
+  a.v_off = 2 * dq;
   a.v_col = rowv ? ws.v_col : nullptr;
   a.v_width = rowv ? ws.v_width : nullptr;
   a.Z = ws.z;
-  a.ld_z = dm;
+  a.ld_z = dq;
   a.z_map = rowv ? wv->row_map : nullptr;
   a.lengths = d->lengths_dev;
   a.batch = d->batch;
   a.seq_len = d->seq_len;
-  a.heads = H;
+  a.heads = Hr;
   a.d_k = dk;
   a.head_begin = 0;
-  a.head_end = H;
+  a.head_end = Hr;
   a.causal = d->causal;
   a.long_form = long_form_for(d) ? 1 : 0;
   a.v_width_max = dk;
@@ -173,18 +188,18 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   a.dtype = d->dtype;
   a.ts = trace_slot(ET_K_ATTN);
   ET_TRY(attention_run(a, st));
-  // 3. output projection -> fp32 (bias and residual are added by the LayerNorm step)
+  // 3. output projection -> partial sums (bias and residual are added by the LayerNorm step)
   GemmArgs o{};
   o.X = ws.z;
   o.M = M;
-  o.K = dm;
-  o.ldx = dm;
+  o.K = dq;
+  o.ldx = dq;
   o.dtype = d->dtype;
   o.nseg = 1;
   o.seg[0] = seg_of(wo, nullptr, 0);
   o.Y = ws.part;
   o.ldy = dm;
-  o.epi = part_epi_of(d->dtype);
+  o.epi = hp ? ET_EPI_F32 : part_epi_of(d->dtype);
   o.ts = trace_slot(ET_K_OPROJ);
   return gemm_run(o, st);
 }
@@ -233,7 +248,7 @@ et_status et_attention_workspace_size(const et_attn_desc* desc, const et_packed_
   if (!wv || !bytes) return fail(ET_ERR_INVALID_ARG, "et_attention_workspace_size: null pointer");
   Carver c{nullptr};
   BlockWs ws;
-  carve_block(c, desc, v_cols_of(wv, desc->d_model), 1, &ws);
+  carve_block(c, desc, v_cols_of(wv, inner_width(desc)), 1, &ws);
   *bytes = c.off + 256;
   return ET_OK;
 }
@@ -244,13 +259,13 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
                            const float* ln_beta, float ln_eps, void* out, void* workspace, size_t ws_bytes,
                            void* stream) {
   ET_TRY(check_desc(desc));
-  if (desc->head_begin != 0 || desc->head_end != desc->heads)
-    return fail(ET_ERR_UNSUPPORTED, "et_attention_fwd: head-parallel ranges are not implemented in this build");
-  const int dm = desc->d_model;
-  ET_TRY(check_weight(wq, dm, dm, desc->dtype, "W_Q", false));
-  ET_TRY(check_weight(wk, dm, dm, desc->dtype, "W_K", false));
-  ET_TRY(check_weight(wv, dm, dm, desc->dtype, "W_V", true));
-  ET_TRY(check_weight(wo, dm, dm, desc->dtype, "W_O", false));
+  const int dm = desc->d_model, dq = inner_width(desc);
+  const bool hp = head_parallel(desc);
+  if (hp && ln_gamma) return fail(ET_ERR_INVALID_ARG, "et_attention_fwd: head-parallel ranges take no LayerNorm (it follows the all-reduce)");
+  ET_TRY(check_weight(wq, dq, dm, desc->dtype, "W_Q", false));
+  ET_TRY(check_weight(wk, dq, dm, desc->dtype, "W_K", false));
+  ET_TRY(check_weight(wv, dq, dm, desc->dtype, "W_V", true));
+  ET_TRY(check_weight(wo, dm, dq, desc->dtype, "W_O", false));
   if (!X || !out || !workspace) return fail(ET_ERR_INVALID_ARG, "et_attention_fwd: null pointer");
   size_t need = 0;
   ET_TRY(et_attention_workspace_size(desc, wv, &need));
@@ -258,14 +273,17 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   Carver c{static_cast<uint8_t*>(workspace)};
   BlockWs ws;
-  carve_block(c, desc, v_cols_of(wv, dm), 1, &ws);
+  carve_block(c, desc, v_cols_of(wv, dq), 1, &ws);
   const void* bo_eff = bo;
   ET_TRY(run_attention_block(desc, X, wq, wk, wv, wo, bq, bk, bv, bo, ws, &bo_eff, st));
   const int M = desc->batch * desc->seq_len;
-  LnArgs ln{ws.part, 1, M, dm, bo_eff, desc->dtype, ln_gamma ? X : nullptr, desc->dtype, ln_gamma, ln_beta, ln_eps,
-            out, nullptr, nullptr, part_dtype_of(desc->dtype)};
+  // full range: out = part + b_O' (+ X and LN when gamma is given), in dtype;
+  // head-parallel: out = FP32 partial (+ b_O' on the rank owning head 0), no residual / LN
+  LnArgs ln{ws.part, 1, M, dm, bo_eff, desc->dtype, ln_gamma ? X : nullptr, hp ? ET_FP32 : desc->dtype, ln_gamma,
+            ln_beta, ln_eps, hp ? nullptr : out, hp ? out : nullptr, nullptr,
+            hp ? ET_FP32 : part_dtype_of(desc->dtype)};
   ln.ts = trace_slot(ET_K_LN1);
-  ET_TRY(layernorm_run(ln, st));   // gamma == NULL: out = attn = part + b_O' (no residual, no LN)
+  ET_TRY(layernorm_run(ln, st));
   return ET_OK;
 }
 
@@ -300,7 +318,8 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
                          size_t ws_bytes, void* stream) {
   ET_TRY(check_desc(desc));
   if (desc->head_begin != 0 || desc->head_end != desc->heads)
-    return fail(ET_ERR_UNSUPPORTED, "et_encoder_fwd: head-parallel ranges are not implemented in this build");
+    return fail(ET_ERR_UNSUPPORTED, "et_encoder_fwd: full head range only (head-parallel layers run as et_attention_fwd "
+                                    "partials + all-reduce + et_layernorm_fwd, dist.HeadParallelEncoder)");
   if (resid_dtype != ET_FP32 && resid_dtype != desc->dtype)
     return fail(ET_ERR_INVALID_ARG, "resid_dtype must be FP32 or the operand dtype");
   if (act != ET_ACT_GELU_ERF && act != ET_ACT_RELU) return fail(ET_ERR_INVALID_ARG, "bad activation");

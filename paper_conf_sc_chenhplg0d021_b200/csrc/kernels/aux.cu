@@ -84,7 +84,7 @@ __global__ void vprep_fold_kernel(const uint8_t* __restrict__ wo_values, const i
       }
     }
   }
-  stf(bo_folded, dt, i, (float)((double)ldf(bo, dt, i) + acc));
+  stf(bo_folded, dt, i, (float)((bo ? (double)ldf(bo, dt, i) : 0.0) + acc));   // bo NULL: fold only (head-parallel rank)
 }
 
 }  // namespace

@@ -87,16 +87,15 @@ __device__ __forceinline__ void layernorm_row(const LnArgs& a) {
     bias[c] = ld_act4<DT>(bias_p, has_bias ? col : 0);
     res[c] = ld_act4<RT>(res_p, has_res ? row + col : 0);
   }
-  const float bsc = has_bias ? 1.0f : 0.0f, rsc = has_res ? 1.0f : 0.0f;
+  // masking by selection, not by multiplying with 0: a dummy read may hold an Inf / NaN bit pattern
+  // (e.g. FP32 partials reinterpreted as 16-bit pairs) and 0 * Inf = NaN
+  auto sel4 = [](bool keep, float4 v) { return keep ? v : make_float4(0.f, 0.f, 0.f, 0.f); };
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
-    const float m = ok[c] ? 1.0f : 0.0f, mb = m * bsc, mr = m * rsc;
 #pragma unroll
-    for (int q = 0; q < NP; ++q) {
-      part[q][c].x *= m; part[q][c].y *= m; part[q][c].z *= m; part[q][c].w *= m;
-    }
-    bias[c].x *= mb; bias[c].y *= mb; bias[c].z *= mb; bias[c].w *= mb;
-    res[c].x *= mr; res[c].y *= mr; res[c].z *= mr; res[c].w *= mr;
+    for (int q = 0; q < NP; ++q) part[q][c] = sel4(ok[c], part[q][c]);
+    bias[c] = sel4(ok[c] && has_bias, bias[c]);
+    res[c] = sel4(ok[c] && has_res, res[c]);
   }
   float4 v[NCH];
   float s = 0.f;
