@@ -43,6 +43,9 @@ typedef enum {
   ET_ERR_INTERNAL = 6
 } et_status;
 
+/* Storage dtypes.  FP16 / BF16: the tcgen05 tensor-core path (FP32 accumulation, reading C-9).
+ * FP32: the validation build (BASELINE configs[0]): every step in FP32 FMA on the CUDA cores
+ * (the 1e-5 gate; one-pass TF32 tensor-core math misses it), packed FP32 tiles row-major, 1 KB. */
 typedef enum { ET_FP16 = 0, ET_BF16 = 1, ET_FP32 = 2 } et_dtype;
 
 /* Pruning patterns (§4.1-4.2; attention-aware assignment line 107, 317). */
@@ -160,7 +163,7 @@ et_status et_layernorm_fwd(const void* part, et_dtype part_dtype, int32_t nparts
 /* ------------------------------------------------------------------------------------------
  * Attention descriptor.
  *   batch, seq_len, heads, d_model   problem statement (d_k = d_model / H)
- *   dtype        storage dtype of activations and weights (FP16 / BF16)
+ *   dtype        storage dtype of activations and weights (FP16 / BF16; FP32 = validation build)
  *   lengths_dev  device int32 [batch], valid length per sequence, 1 <= len <= seq_len; keys
  *                j >= len are masked (probability exactly 0, line 73; reading C-7).  NULL = all.
  *   causal       nonzero: also mask j > i (the triangular mask of line 73)

@@ -157,9 +157,9 @@ et_status et_prune_pack_query(int32_t rows, int32_t cols, et_dtype dtype, et_pat
   if (tilecol_bytes) *tilecol_bytes = (size_t)(tiles_max > 0 ? tiles_max : 1) * 4 + 16;   // +16: aligned bulk reads
   if (rowmap_bytes) *rowmap_bytes = pattern == ET_PRUNE_ROW ? (size_t)tile_rows_max * 16 * 4 : 4;
   if (partrowptr_bytes) *partrowptr_bytes = (size_t)kparts * (tile_rows_max + 1) * 4;
-  const bool has_values = tile_r == 16 && tile_c == 16 && dtype != ET_FP32 && pattern != ET_PRUNE_COL &&
-                          cols % 16 == 0;
-  if (values_bytes) *values_bytes = has_values ? (size_t)(tiles_max > 0 ? tiles_max : 1) * 512 : 0;
+  const bool has_values = tile_r == 16 && tile_c == 16 && pattern != ET_PRUNE_COL && cols % 16 == 0;
+  // 16-bit tiles: 512 B in the tcgen05 core-matrix layout; FP32 tiles: 1 KB row-major (simt32.cu)
+  if (values_bytes) *values_bytes = has_values ? (size_t)(tiles_max > 0 ? tiles_max : 1) * 256 * dtype_size(dtype) : 0;
   if (workspace_bytes) *workspace_bytes = prune_workspace_bytes(rows, cols, pattern, tile_r, tile_c);
   return ET_OK;
 }

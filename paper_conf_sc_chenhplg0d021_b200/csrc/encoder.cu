@@ -45,8 +45,8 @@ et_status check_desc(const et_attn_desc* d) {
   if (d->batch <= 0 || d->seq_len <= 0 || d->heads <= 0 || d->d_model <= 0)
     return fail(ET_ERR_INVALID_ARG, "batch, seq_len, heads, d_model must be positive");
   if (d->d_model % d->heads) return fail(ET_ERR_INVALID_ARG, "d_model %% heads != 0");
-  if (d->dtype != ET_FP16 && d->dtype != ET_BF16)
-    return fail(ET_ERR_UNSUPPORTED, "forward path: dtype must be FP16 or BF16 in this build");
+  if (d->dtype != ET_FP16 && d->dtype != ET_BF16 && d->dtype != ET_FP32)
+    return fail(ET_ERR_INVALID_ARG, "forward path: dtype must be FP16, BF16 or FP32 (validation build)");
   const int dk = d->d_model / d->heads;
   if (dk != 64 && dk != 128) return fail(ET_ERR_UNSUPPORTED, "d_k must be 64 or 128 (got %d)", dk);
   if (d->d_model % 64) return fail(ET_ERR_UNSUPPORTED, "d_model must be a multiple of 64");

@@ -74,6 +74,8 @@ struct GemmArgs {
   unsigned long long* ts;   // trace slot or nullptr
 };
 et_status gemm_run(const GemmArgs& a, cudaStream_t stream);
+// FP32 validation build (kernels/simt32.cu): CUDA-core FP32 FMA, same arguments
+et_status gemm32_run(const GemmArgs& a, cudaStream_t stream);
 
 // ---------------------------------------------------------------- LayerNorm (kernels/layernorm.cu)
 struct LnArgs {
@@ -112,6 +114,7 @@ struct AttnArgs {
   unsigned long long* ts;   // trace slot or nullptr
 };
 et_status attention_run(const AttnArgs& a, cudaStream_t stream);
+et_status attention32_run(const AttnArgs& a, cudaStream_t stream);
 // seq_len <= 128, d_k = 64, dense V: the 3-CTAs-per-SM kernel (kernels/attention128.cu)
 bool attention128_applies(const AttnArgs& a);
 et_status attention128_run(const AttnArgs& a, cudaStream_t stream);

@@ -496,7 +496,7 @@ et_status launch(const CUtensorMap& tm, const CUtensorMap& tz, const AParams& pr
 int attn_short_max(int d_k) { return (d_k == 64 || d_k == 128) ? 256 : 0; }
 
 et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
-  if (a.dtype == ET_FP32) return fail(ET_ERR_UNSUPPORTED, "attention: FP32 not implemented in this build");
+  if (a.dtype == ET_FP32) return attention32_run(a, stream);   // FP32 validation build (CUDA cores)
   if (a.d_k != 64 && a.d_k != 128) return fail(ET_ERR_UNSUPPORTED, "attention: d_k must be 64 or 128 (got %d)", a.d_k);
   if (a.v_width_max <= 0 || a.v_width_max > a.d_k || a.v_width_max % 16)
     return fail(ET_ERR_INVALID_ARG, "attention: V width must be a multiple of 16 and <= d_k");

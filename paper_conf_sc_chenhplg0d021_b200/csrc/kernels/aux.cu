@@ -72,14 +72,17 @@ __global__ void vprep_fold_kernel(const uint8_t* __restrict__ wo_values, const i
     const int32_t* rp = wo_prp + z * (wo_tile_rows + 1);
     for (int t = rp[ti]; t < rp[ti + 1]; ++t) {
       const int j = wo_tile_col[t];
-      const uint8_t* tile = wo_values + (size_t)t * 512;
+      const uint8_t* tile = wo_values + (size_t)t * 256 * (dt == ET_FP32 ? 4 : 2);
       for (int k = 0; k < 16; ++k) {
         const int f = j * 16 + k;
         if ((wv_mask[f >> 5] >> (f & 31)) & 1u) continue;   // kept V feature: no fold
-        const uint16_t raw = *reinterpret_cast<const uint16_t*>(tile + (n >> 3) * 256 + (k >> 3) * 128 + (n & 7) * 16 + (k & 7) * 2);
         float w;
-        if (dt == ET_BF16) w = __bfloat162float(__ushort_as_bfloat16(raw));
-        else w = __half2float(__ushort_as_half(raw));
+        if (dt == ET_FP32) {   // FP32 tiles: row-major (simt32.cu)
+          w = *reinterpret_cast<const float*>(tile + n * 64 + k * 4);
+        } else {
+          const uint16_t raw = *reinterpret_cast<const uint16_t*>(tile + (n >> 3) * 256 + (k >> 3) * 128 + (n & 7) * 16 + (k & 7) * 2);
+          w = dt == ET_BF16 ? __bfloat162float(__ushort_as_bfloat16(raw)) : __half2float(__ushort_as_half(raw));
+        }
         acc += (double)w * (double)ldf(bv, dt, f);
       }
     }

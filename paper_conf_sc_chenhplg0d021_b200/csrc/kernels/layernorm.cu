@@ -190,6 +190,8 @@ et_status launch_dt(const LnArgs& a, cudaStream_t stream) {
     return p16 ? launch_np<NCH, ET_BF16, ET_BF16, true>(a, stream) : launch_np<NCH, ET_BF16, ET_BF16, false>(a, stream);
   if (dt == ET_BF16 && rt == ET_FP32)
     return p16 ? launch_np<NCH, ET_BF16, ET_FP32, true>(a, stream) : launch_np<NCH, ET_BF16, ET_FP32, false>(a, stream);
+  if (dt == ET_FP32 && rt == ET_FP32 && !p16)   // FP32 validation build
+    return launch_np<NCH, ET_FP32, ET_FP32, false>(a, stream);
   return fail(ET_ERR_UNSUPPORTED, "LayerNorm: dtype pair (%d, %d) not supported", dt, rt);
 }
 

@@ -222,6 +222,50 @@ __global__ void pack_values_kernel(const uint16_t* __restrict__ W, int cols, int
   *reinterpret_cast<uint4*>(values + (size_t)warp * 512 + (n >> 3) * 256 + kh * 128 + (n & 7) * 16) = v;
 }
 
+// FP32 validation build: the same tile order, each tile row-major (element (n, k) at byte
+// n*64 + k*4, 1 KB).  Lane l moves row n = l/2, half kh = l%2 (8 floats).
+__global__ void pack_values32_kernel(const float* __restrict__ W, int cols, int pattern,
+                                     const int32_t* __restrict__ part_row_ptr, const int32_t* __restrict__ tile_col,
+                                     const int32_t* __restrict__ row_map, const int32_t* __restrict__ counts,
+                                     int kparts, float* __restrict__ values, int rows) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int ntiles = counts[2];
+  if (warp >= ntiles) return;
+  const int tile_rows = pattern == ET_PRUNE_TILE ? rows / 16 : counts[1] / 16;
+  const int i = tile_row_of(part_row_ptr, tile_rows, kparts, warp);
+  const int j = tile_col[warp];
+  const int n = lane >> 1, kh = lane & 1;
+  const int src_row = pattern == ET_PRUNE_TILE ? i * 16 + n : row_map[i * 16 + n];
+  float4 a = make_float4(0.f, 0.f, 0.f, 0.f), b = a;
+  if (src_row >= 0) {
+    const float4* s = reinterpret_cast<const float4*>(W + (size_t)src_row * cols + j * 16 + kh * 8);
+    a = s[0];
+    b = s[1];
+  }
+  float4* d = reinterpret_cast<float4*>(values + (size_t)warp * 256 + n * 16 + kh * 8);
+  d[0] = a;
+  d[1] = b;
+}
+
+__global__ void unpack32_kernel(const float* __restrict__ values, int cols, int pattern,
+                                const int32_t* __restrict__ part_row_ptr, const int32_t* __restrict__ tile_col,
+                                const int32_t* __restrict__ row_map, int ntiles, int tile_rows, int kparts,
+                                float* __restrict__ dense) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (warp >= ntiles) return;
+  const int i = tile_row_of(part_row_ptr, tile_rows, kparts, warp);
+  const int j = tile_col[warp];
+  const int n = lane >> 1, kh = lane & 1;
+  const int dst_row = pattern == ET_PRUNE_TILE ? i * 16 + n : row_map[i * 16 + n];
+  if (dst_row < 0) return;
+  const float4* s = reinterpret_cast<const float4*>(values + (size_t)warp * 256 + n * 16 + kh * 8);
+  float4* d = reinterpret_cast<float4*>(dense + (size_t)dst_row * cols + j * 16 + kh * 8);
+  d[0] = s[0];
+  d[1] = s[1];
+}
+
 // Inverse of pack_values_kernel: dense [rows, cols] = 0 except kept tiles / rows.
 __global__ void unpack_kernel(const uint8_t* __restrict__ values, int cols, int pattern,
                               const int32_t* __restrict__ part_row_ptr, const int32_t* __restrict__ tile_col,
@@ -293,8 +337,7 @@ et_status prune_pack_run(const PruneArgs& a, et_packed_weight* out, void* ws, si
                                      out->row_ptr, out->tile_col, out->row_map, out->part_row_ptr, counts);
   count_launch();
   ET_CUDA(cudaGetLastError());
-  const bool pack_values = out->values != nullptr && a.dtype != ET_FP32 && a.tile_r == 16 && a.tile_c == 16 &&
-                           a.pattern != ET_PRUNE_COL;
+  const bool pack_values = out->values != nullptr && a.tile_r == 16 && a.tile_c == 16 && a.pattern != ET_PRUNE_COL;
   const int kparts = (a.cols / 16 + 47) / 48;
   if (pack_values) {
     if (!out->tile_col || !out->part_row_ptr || (a.pattern == ET_PRUNE_ROW && !out->row_map))
@@ -304,9 +347,14 @@ et_status prune_pack_run(const PruneArgs& a, et_packed_weight* out, void* ws, si
     const int max_tiles = a.pattern == ET_PRUNE_TILE ? units : ((a.rows + 15 * groups) / 16 + 1) * (a.cols / 16);
     const int threads = 256;
     const int blocks = (max_tiles * 32 + threads - 1) / threads;
-    pack_values_kernel<<<blocks, threads, 0, stream>>>(static_cast<const uint16_t*>(a.W), a.cols, a.pattern,
-                                                       out->part_row_ptr, out->tile_col, out->row_map, counts,
-                                                       kparts, static_cast<uint8_t*>(out->values), a.rows);
+    if (a.dtype == ET_FP32)
+      pack_values32_kernel<<<blocks, threads, 0, stream>>>(static_cast<const float*>(a.W), a.cols, a.pattern,
+                                                           out->part_row_ptr, out->tile_col, out->row_map, counts,
+                                                           kparts, static_cast<float*>(out->values), a.rows);
+    else
+      pack_values_kernel<<<blocks, threads, 0, stream>>>(static_cast<const uint16_t*>(a.W), a.cols, a.pattern,
+                                                         out->part_row_ptr, out->tile_col, out->row_map, counts,
+                                                         kparts, static_cast<uint8_t*>(out->values), a.rows);
   count_launch();
     ET_CUDA(cudaGetLastError());
   }
@@ -321,12 +369,21 @@ et_status prune_pack_run(const PruneArgs& a, et_packed_weight* out, void* ws, si
 }
 
 et_status unpack_run(const et_packed_weight* w, void* dense, cudaStream_t stream) {
-  if (w->values == nullptr || w->dtype == ET_FP32)
-    return fail(ET_ERR_UNSUPPORTED, "et_unpack: no packed values (FP32 or non-16x16 tiles)");
-  ET_CUDA(cudaMemsetAsync(dense, 0, (size_t)w->rows * w->cols * 2, stream));
+  if (w->values == nullptr)
+    return fail(ET_ERR_UNSUPPORTED, "et_unpack: no packed values (non-16x16 tiles or column pattern)");
+  ET_CUDA(cudaMemsetAsync(dense, 0, (size_t)w->rows * w->cols * dtype_size(w->dtype), stream));
   if (w->ntiles == 0) return ET_OK;
   const int threads = 256;
   const int blocks = (w->ntiles * 32 + threads - 1) / threads;
+  if (w->dtype == ET_FP32) {
+    unpack32_kernel<<<blocks, threads, 0, stream>>>(static_cast<const float*>(w->values), w->cols, w->pattern,
+                                                    w->part_row_ptr, w->tile_col, w->row_map, w->ntiles,
+                                                    w->pattern == ET_PRUNE_TILE ? w->rows / 16 : w->rows_padded / 16,
+                                                    w->kparts, static_cast<float*>(dense));
+    count_launch();
+    ET_CUDA(cudaGetLastError());
+    return ET_OK;
+  }
   unpack_kernel<<<blocks, threads, 0, stream>>>(static_cast<const uint8_t*>(w->values), w->cols, w->pattern,
                                                 w->part_row_ptr, w->tile_col, w->row_map, w->ntiles,
                                                 w->pattern == ET_PRUNE_TILE ? w->rows / 16 : w->rows_padded / 16,

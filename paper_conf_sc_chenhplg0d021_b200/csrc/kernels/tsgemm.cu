@@ -642,7 +642,7 @@ et_status make_tmap_3d(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t col
 }
 
 et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
-  if (a.dtype == ET_FP32) return fail(ET_ERR_UNSUPPORTED, "tile GEMM: FP32 operands not implemented in this build");
+  if (a.dtype == ET_FP32) return gemm32_run(a, stream);   // FP32 validation build (CUDA cores)
   if (a.K % 64) return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K must be a multiple of 64 (got %d)", a.K);
   if (!aligned16(a.X) || (a.ldx * 2) % 16 || (a.k0 * 2) % 16)
     return fail(ET_ERR_INVALID_ARG, "tile GEMM: X must be 16-byte aligned with 16-byte row pitch");

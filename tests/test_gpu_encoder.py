@@ -1,6 +1,6 @@
 """End-to-end parity of et_encoder_fwd / et_attention_fwd vs the float64 oracle:
-every BASELINE config shape (C1..C5; C1 in FP16/BF16 — the FP32 validation build is not in this
-build), reduced and at full size on sampled sequences, both residual-stream dtypes, and the
+every BASELINE config shape (C1..C5; C1 also in FP16/BF16 here — its FP32 validation build is
+tested in test_gpu_fp32.py), reduced and at full size on sampled sequences, both residual-stream dtypes, and the
 batch-shard bit-exactness that multi-GPU batch sharding relies on (§8(e))."""
 import numpy as np
 import pytest
