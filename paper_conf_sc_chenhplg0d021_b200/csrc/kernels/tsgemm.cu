@@ -82,7 +82,8 @@ constexpr int kSlotBytes = 16384;
 constexpr int kChunkTiles = 32;  // tiles per tile chunk (16 KB)
 constexpr int kMaxKChunks = 12;  // K <= 768 per part
 constexpr int kMaxBChunks = 192; // tile chunks per CTA (one single-use full barrier each)
-constexpr int kMaxRows = 256;    // tile rows per CTA (row pointers and bias staged in smem)
+constexpr int kMaxRows = 256;    // tile rows per CTA (row pointers staged in smem)
+constexpr int kMaxBiasRows = 128; // tile rows per CTA of a bias epilogue (FP32 bias staged in smem)
 constexpr int kAccCol = 384;     // first accumulator column (A uses [0, Kp/2) <= 384)
 constexpr int kMmaWarps = 8;     // warps 0-7: MMA issue, one accumulator (16 TMEM columns) each
 constexpr int kEpiGroups = 4;    // warps 8-23: epilogue, 4 groups of 4 (one warp per TMEM lane quarter);
@@ -133,7 +134,7 @@ struct __align__(16) Barriers {
   uint64_t bfull[kMaxBChunks];
   alignas(16) int tcol[kMaxSlots][kChunkTiles + 4];   // bulk-copy destination (16-byte aligned): tile columns
   int rptr[kMaxRows + 1];        // this CTA's row pointers, relative to its first tile
-  uint32_t bias_s[kMaxRows * 8]; // this CTA's bias slice (16-bit pairs)
+  alignas(16) float bias_f[kMaxBiasRows * 16];   // this CTA's bias slice, FP32 (converted once)
   uint32_t tmem_base;
   int rows_seen[kEpiGroups];     // per epilogue group: rows whose MMAs were observed complete (in order)
   int tcoff[kMaxSlots];          // per slot: offset of the chunk's first column index in tcol[slot]
@@ -211,7 +212,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int nrows = rowsA + rowsB;
   const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
 
-  if (nchunks > kMaxBChunks || nrows > kMaxRows) __trap();   // host sizes pieces so this cannot happen
+  if (nchunks > kMaxBChunks || nrows > kMaxRows || (!is_partial(kEpi) && nrows > kMaxBiasRows))
+    __trap();   // host sizes pieces so this cannot happen
   // A chunks are loaded in K order (the first round's MMAs follow the fill chunk by chunk).
   // ET_GEMM_A_ROT: rotate the order per piece instead (CTAs of one token block start a quarter of
   // the block apart) — measured no faster: the L2 serves the sharing CTAs well (profiles/r01).
@@ -320,7 +322,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
 #pragma unroll
             for (int g = 0; g < kEpiGroups; ++g) {
               const int need = 2 * full + min(max(rem - 2 * g, 0), 2);
-              while (ld_acquire_shared(&bar.rows_seen[g]) < need) {}
+              while (ld_acquire_shared(&bar.rows_seen[g]) < need) {}   // (a __nanosleep back-off made every GEMM slower)
             }
           }
         }
@@ -421,7 +423,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         const int t = i >> 3;
         const uint32_t* bsrc = static_cast<const uint32_t*>(t < rowsA ? sa.bias : sb.bias);
         const int row = t < rowsA ? pc.i0 + t : t - rowsA;
-        bar.bias_s[i] = bsrc ? __ldg(bsrc + (size_t)row * 8 + (i & 7)) : 0u;
+        const float2 f = unpack2<kBF16>(bsrc ? __ldg(bsrc + (size_t)row * 8 + (i & 7)) : 0u);
+        *reinterpret_cast<float2*>(&bar.bias_f[2 * i]) = f;
       }
       named_bar_sync(1, kEpiWarps * 32);
     }
@@ -453,19 +456,23 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
 #pragma unroll
       for (int a = 0; a < 2; ++a) {
         const int t = t0 + min(a, na - 1);
+        // a row with no kept tile was never written: its accumulator is zero (output = epi(bias))
         const bool empty_row = a >= na || rend(t) == bar.rptr[t];
+        const float4* bt = reinterpret_cast<const float4*>(&bar.bias_f[(is_partial(kEpi) ? 0 : t) * 16]);
+        float sc = 1.0f;
+        if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
+          const SegDev& st_seg = t < rowsA ? sa : sb;
+          if (st_seg.apply_scale) sc = st_seg.scale;
+        }
 #pragma unroll
         for (int c = 0; c < 16; c += 2) {
-          // a row with no kept tile was never written: its accumulator is zero (output = epi(bias))
           float x0 = empty_row ? 0.0f : __uint_as_float(r[a * 16 + c]);
           float x1 = empty_row ? 0.0f : __uint_as_float(r[a * 16 + c + 1]);
           if constexpr (!is_partial(kEpi)) {
-            const float2 bb = unpack2<kBF16>(bar.bias_s[t * 8 + c / 2]);
+            const float4 b4 = bt[c / 4];   // broadcast LDS.128, shared by every thread of the group
+            const float2 bb = (c & 2) ? make_float2(b4.z, b4.w) : make_float2(b4.x, b4.y);
             uint64_t xx = fadd2(f2pk(x0, x1), f2pk(bb.x, bb.y));
-            if constexpr (kEpi == ET_EPI_BIAS_SCALE) {
-              const SegDev& st_seg = t < rowsA ? sa : sb;
-              if (st_seg.apply_scale) xx = fmul2(xx, f2pk(st_seg.scale, st_seg.scale));
-            }
+            if constexpr (kEpi == ET_EPI_BIAS_SCALE) xx = fmul2(xx, f2pk(sc, sc));
             const float2 xf = f2upk(xx);
             x0 = xf.x;
             x1 = xf.y;
@@ -684,7 +691,8 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     prm.seg[s].apply_scale = gs.apply_scale;
   }
   const int kt = std::min(a.K, 768) / 16;   // tile columns per K part (bound on tiles per row)
-  auto fits = [&](int rows) { return rows <= kMaxRows && (long long)rows * kt + kChunkTiles <= (long long)kMaxBChunks * kChunkTiles; };
+  const int max_rows = is_partial(a.epi) ? kMaxRows : kMaxBiasRows;
+  auto fits = [&](int rows) { return rows <= max_rows && (long long)rows * kt + kChunkTiles <= (long long)kMaxBChunks * kChunkTiles; };
   int np = 0;
   // Output-contiguous segments (Q|K|V): plan the pieces over the concatenated tile rows, so the CTA
   // count is set by the total rows rather than rounded per segment (4 pieces of 36 rows instead of
