@@ -72,7 +72,17 @@ struct GemmArgs {
   int ldy;
   et_epilogue epi;
   unsigned long long* ts;   // trace slot or nullptr
+  // kEpiLN (fused residual + LayerNorm, internal): Y = LN(acc + b + resid) * gamma + beta
+  const void* resid;        // [M, ldy] in dtype
+  const float* gamma;
+  const float* beta;
+  float eps;
 };
+// internal epilogue id (not in the public et_epilogue): residual + LayerNorm fused into the GEMM,
+// row statistics exchanged across the cluster of CTAs sharing a token block (DSMEM)
+constexpr int kEpiLN = 16;
+// true if gemm_run can run `a` with kEpiLN (shape / dtype / piece constraints)
+bool gemm_ln_applies(const GemmArgs& a);
 et_status gemm_run(const GemmArgs& a, cudaStream_t stream);
 // FP32 validation build (kernels/simt32.cu): CUDA-core FP32 FMA, same arguments
 et_status gemm32_run(const GemmArgs& a, cudaStream_t stream);
@@ -163,6 +173,26 @@ cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t sme
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+// The same with a thread-block cluster of (cluster_x, 1, 1) CTAs (grid.x must be a multiple).
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
+                               unsigned cluster_x, Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  attr[1].id = cudaLaunchAttributeClusterDimension;
+  attr[1].val.clusterDim.x = cluster_x;
+  attr[1].val.clusterDim.y = 1;
+  attr[1].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 2;
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }   // device slot of the next traced launch, or nullptr
 void count_launch();
