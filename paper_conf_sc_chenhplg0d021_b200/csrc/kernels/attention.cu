@@ -81,6 +81,13 @@ struct Cfg {
   static constexpr int kHalf = kDK / 2;              // O columns per softmax thread
   static constexpr int kStageBytes = 32 * kHalf * 2; // per softmax warp: 32 rows x kHalf fp16
 };
+// K/V ring depth: the short form holds all (<= 2) key blocks; the long form streams them through 4
+// stages at d_k = 64 (the K/V load of block j+4 overlaps three blocks of work; with 2 stages the
+// load of block j+2 could only start once P.V(j) had completed), 2 at d_k = 128 (shared memory)
+template <bool kLong, int kDK> constexpr int kv_stages() { return (kLong && kDK == 64) ? 4 : 2; }
+template <bool kLong, int kDK> constexpr size_t attn_smem_bytes() {
+  return 1024 + (size_t)(1 + 2 * kv_stages<kLong, kDK>()) * Cfg<kDK>::kOpBytes + 8 * Cfg<kDK>::kStageBytes + 2048 + 256;
+}
 
 __device__ __forceinline__ float ex2(float x) {
   float y;
@@ -98,6 +105,7 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
                                                            const __grid_constant__ CUtensorMap tmap_z,
                                                            const __grid_constant__ AParams p) {
   using C = Cfg<kDK>;
+  constexpr int kKV = kv_stages<kLong, kDK>();
   constexpr int kS = 0, kP = 128 * kNKB, kO = 192 * kNKB;
   constexpr uint32_t kCols = (kO + kDK) <= 256 ? 256u : 512u;
   pdl_trigger();
@@ -112,21 +120,21 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
   // address space (an integer round trip would turn every access into a generic LD/ST)
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sQ = smem;
-  uint8_t* sK = sQ + C::kOpBytes;                // 2 x K block
-  uint8_t* sV = sK + 2 * C::kOpBytes;            // 2 x V block
-  uint8_t* sStage = sV + 2 * C::kOpBytes;        // 8 x epilogue staging
+  uint8_t* sK = sQ + C::kOpBytes;                // kKV x K block
+  uint8_t* sV = sK + kKV * C::kOpBytes;          // kKV x V block
+  uint8_t* sStage = sV + kKV * C::kOpBytes;      // 8 x epilogue staging
   float* xmax = reinterpret_cast<float*>(sStage + 8 * C::kStageBytes);   // [2][128] row-max halves
   float* xsum = xmax + 256;                                               // [2][128] row-sum halves
   uint64_t* bars = reinterpret_cast<uint64_t*>(xsum + 256);
   uint64_t* q_full = bars + 0;
-  uint64_t* kv_full = bars + 1;       // [2]
-  uint64_t* kv_empty = bars + 3;      // [2]
-  uint64_t* s_full = bars + 5;        // [2]
-  uint64_t* s_free = bars + 7;        // [2]
-  uint64_t* p_full = bars + 9;        // [2]
-  uint64_t* o_full = bars + 11;
-  uint64_t* o_free = bars + 12;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
+  uint64_t* kv_full = bars + 1;              // [kKV]
+  uint64_t* kv_empty = bars + 1 + kKV;       // [kKV]
+  uint64_t* s_full = bars + 1 + 2 * kKV;     // [2]
+  uint64_t* s_free = s_full + 2;             // [2]
+  uint64_t* p_full = s_full + 4;             // [2]
+  uint64_t* o_full = s_full + 6;
+  uint64_t* o_free = s_full + 7;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(s_full + 8);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -148,15 +156,17 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
   if (p.box_rows < 128) {
     // tiny problem: the TMA box covers fewer than 128 rows; zero the V staging so that the rows
     // it leaves untouched are finite (P = 0 there, but 0 * NaN would poison O)
-    for (int i = threadIdx.x; i < 2 * C::kOpBytes / 16; i += blockDim.x)
+    for (int i = threadIdx.x; i < kKV * C::kOpBytes / 16; i += blockDim.x)
       reinterpret_cast<uint4*>(sV)[i] = make_uint4(0, 0, 0, 0);
     fence_proxy_async_smem();
   }
   if (threadIdx.x == 0) {
     mbar_init(q_full, 1);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < kKV; ++i) {
       mbar_init(&kv_full[i], 1);
       mbar_init(&kv_empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
       mbar_init(&s_full[i], 1);
       mbar_init(&s_free[i], 8);
       mbar_init(&p_full[i], 8);
@@ -182,8 +192,8 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
       for (int t = 0; t < C::kTiles; ++t)
         tma_load_2d(sQ + t * 16384, &tmap, q_full, qcol + t * 64, row0 + qb * 128);
       for (int j = 0; j < nkb; ++j) {
-        const int st = j & 1;
-        if (j >= 2) mbar_wait(&kv_empty[st], ((j >> 1) - 1) & 1);
+        const int st = j % kKV;
+        if (j >= kKV) mbar_wait(&kv_empty[st], ((j / kKV) - 1) & 1);
         mbar_expect_tx(&kv_full[st], 2 * tile_bytes * C::kTiles);
         for (int t = 0; t < C::kTiles; ++t) {
           tma_load_2d(sK + st * C::kOpBytes + t * 16384, &tmap, &kv_full[st], kcol + t * 64, row0 + j * 128);
@@ -197,7 +207,7 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
     const uint32_t idesc_o = make_idesc_f16(128, dvn, kBF16 ? 1 : 0, 0, 1);          // P.V, V MN-major
     const uint32_t q_u = smem_u32(sQ);
     auto issue_qk = [&](int j, uint32_t s_col) {
-      const uint32_t k_u = smem_u32(sK + (j & 1) * C::kOpBytes);
+      const uint32_t k_u = smem_u32(sK + (j % kKV) * C::kOpBytes);
 #pragma unroll
       for (int ks = 0; ks < kDK / 16; ++ks) {
         const uint32_t off = (ks >> 2) * 16384 + (ks & 3) * 32;
@@ -206,7 +216,7 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
       }
     };
     auto issue_pv = [&](int j, uint32_t p_col, bool acc_first) {
-      const uint32_t v_u = smem_u32(sV + (j & 1) * C::kOpBytes);
+      const uint32_t v_u = smem_u32(sV + (j % kKV) * C::kOpBytes);
 #pragma unroll
       for (int ks = 0; ks < 8; ++ks)   // 128 keys = 8 x K16; V MN-major SW128: 16 rows = 2048 B
         mma_ts_warp(tbase + kO, tbase + p_col + ks * 8, make_sdesc(v_u + ks * 2048, 16384, 1024, kLayoutSW128),
@@ -241,17 +251,16 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
         if (j + 1 < nkb) {
           const int jn = j + 1, bn = jn & 1;
           if (jn >= 2) mbar_wait_warp(&s_free[bn], ((jn >> 1) - 1) & 1);
-          mbar_wait_warp(&kv_full[bn], (jn >> 1) & 1);
+          mbar_wait_warp(&kv_full[jn % kKV], (jn / kKV) & 1);
           tc_fence_after();
           issue_qk(jn, kS + bn * 128);
           mma_commit_warp(&s_full[bn]);
         }
         mbar_wait_warp(&p_full[j & 1], (j >> 1) & 1);
-        if (j >= 1) mbar_wait_warp(o_free, (j - 1) & 1);
         tc_fence_after();
-        issue_pv(j, kP + (j & 1) * 64, false);
+        issue_pv(j, kP + (j & 1) * 64, j > 0);   // O accumulates in TMEM (rescaled there when needed)
         mma_commit_warp(o_full);
-        mma_commit_warp(&kv_empty[j & 1]);
+        mma_commit_warp(&kv_empty[j % kKV]);
       }
     }
   } else {
@@ -266,9 +275,6 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
     int kend = len;                              // valid keys: [0, kend)
     if (p.causal) kend = min(kend, qi + 1);
     const float sl2 = p.scale_log2;
-    float o[kLong ? C::kHalf : 1];
-#pragma unroll
-    for (int c = 0; c < (kLong ? C::kHalf : 1); ++c) o[c] = 0.f;
     float lpart = 0.f;                           // this half's share of the row sum
 
     if constexpr (!kLong) {
@@ -319,76 +325,100 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
       tc_fence_after();
       if (threadIdx.x == 64) ET_TLA(7);
     } else {
-      float m = -INFINITY;
+      // Per 128-key block: the half-row of scores is read from TMEM ONCE into registers (the S
+      // buffer is released at once for QK(j+2)), max and exp2 come from the registers.  O stays in
+      // TMEM and accumulates across blocks; it is rescaled there only when a row's running max grows
+      // by more than 2^8 in exp2 units (otherwise the stale max is kept: p <= 2^8, exact in the
+      // final O / l since l uses the same max — lazy rescaling as in FlashAttention-4).
+      constexpr float kRescale = 8.0f;
+      float m = -INFINITY;                       // max used for this row's exponentials so far
       for (int j = 0; j < nkb; ++j) {
         const int bj = j & 1;
         mbar_wait_warp(&s_full[bj], (j >> 1) & 1);
         tc_fence_after();
-        // pass A: block max over this half's valid keys, combined with the other half
-        float mblk = -INFINITY;
+        uint32_t sv0[32], sv1[32];
+        tmem_ld32(tbase + lane_off + kS + bj * 128 + half * 64, sv0);
+        tmem_ld32(tbase + lane_off + kS + bj * 128 + half * 64 + 32, sv1);
+        tmem_ld_wait();
+        auto sv = [&](int t) { return t < 32 ? sv0[t] : sv1[t - 32]; };
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&s_free[bj]);   // S(j) is in registers: its buffer may take QK(j+2)
+        const int kb = j * 128 + half * 64;        // first key of this thread's half block
+        const bool full = kb + 64 <= kend;         // no masked key in this half block
+        // 8 independent partial maxima / sums: the reductions are not one 64-long dependency chain
+        float mx8[8];
 #pragma unroll
-        for (int c = 0; c < 2; ++c) {
-          uint32_t v[32];
-          const int kl = half * 64 + c * 32;
-          tmem_ld32(tbase + lane_off + kS + bj * 128 + kl, v);
-          tmem_ld_wait();
+        for (int i = 0; i < 8; ++i) mx8[i] = -INFINITY;
+        if (full) {
 #pragma unroll
-          for (int t = 0; t < 32; ++t)
-            if (j * 128 + kl + t < kend) mblk = fmaxf(mblk, __uint_as_float(v[t]));
+          for (int t = 0; t < 64; ++t) mx8[t & 7] = fmaxf(mx8[t & 7], __uint_as_float(sv(t)));
+        } else {
+#pragma unroll
+          for (int t = 0; t < 64; ++t)
+            if (kb + t < kend) mx8[t & 7] = fmaxf(mx8[t & 7], __uint_as_float(sv(t)));
         }
+        float mblk = fmaxf(fmaxf(fmaxf(mx8[0], mx8[1]), fmaxf(mx8[2], mx8[3])),
+                           fmaxf(fmaxf(mx8[4], mx8[5]), fmaxf(mx8[6], mx8[7])));
         xmax[half * 128 + r] = mblk;
         named_bar_sync(1, 256);
         mblk = fmaxf(mblk, xmax[(half ^ 1) * 128 + r]);
         named_bar_sync(2, 256);   // both halves read xmax before it is rewritten for the next block
-        const float m_new = fmaxf(m, mblk);
-        const float alpha = (m == -INFINITY) ? 0.f : ex2((m - m_new) * sl2);
-        const float mb = m_new * sl2;
-        float lsum = 0.f;
-        // pass B: p = exp(s - m_new) -> P(j) in TMEM buffer j&1 (its previous reader PV(j-2)
-        // completed before o_full(j-1) was observed)
+        float alpha = 1.0f;
+        if (mblk > m && (m == -INFINITY || (mblk - m) * sl2 > kRescale)) {
+          alpha = (m == -INFINITY) ? 0.f : ex2((m - mblk) * sl2);
+          m = mblk;
+        }
+        // PV(j-1) must be complete before O is rescaled and before P buffer bj (read by PV(j-2))
+        // is overwritten (in-order completion: o_full phase j-1 covers both)
+        if (j >= 1) {
+          mbar_wait_warp(o_full, (j - 1) & 1);
+          tc_fence_after();
+          if (__any_sync(0xffffffffu, alpha != 1.0f)) {   // warp-collective TMEM read-modify-write
+#pragma unroll
+            for (int c = 0; c < C::kHalf; c += 32) {
+              if (half * C::kHalf + c < dvn) {
+                uint32_t ov[32];
+                tmem_ld32(tbase + lane_off + kO + half * C::kHalf + c, ov);
+                tmem_ld_wait();
+#pragma unroll
+                for (int t = 0; t < 32; ++t) ov[t] = __float_as_uint(__uint_as_float(ov[t]) * alpha);
+                tmem_st32(tbase + lane_off + kO + half * C::kHalf + c, ov);
+              }
+            }
+          }
+        }
+        const float mb = (m == -INFINITY) ? 0.f : m * sl2;
+        uint64_t ls4[4] = {0ull, 0ull, 0ull, 0ull};   // 4 packed FP32x2 partial sums
+        const uint64_t sl2x2 = f2pk(sl2, sl2), nmb2 = f2pk(-mb, -mb);
 #pragma unroll
         for (int c = 0; c < 2; ++c) {
-          uint32_t v[32];
-          const int kl = half * 64 + c * 32;
-          tmem_ld32(tbase + lane_off + kS + bj * 128 + kl, v);
-          tmem_ld_wait();
           uint32_t pk[16];
 #pragma unroll
           for (int t = 0; t < 32; t += 2) {
-            const int key = j * 128 + kl + t;
-            const float p0 = key < kend ? ex2(__uint_as_float(v[t]) * sl2 - mb) : 0.f;
-            const float p1 = key + 1 < kend ? ex2(__uint_as_float(v[t + 1]) * sl2 - mb) : 0.f;
-            lsum += p0 + p1;
+            const int key = kb + c * 32 + t;
+            const float2 x = f2upk(ffma2(f2pk(__uint_as_float(sv(c * 32 + t)), __uint_as_float(sv(c * 32 + t + 1))),
+                                         sl2x2, nmb2));   // s * scale * log2 e - m * scale * log2 e
+            float p0 = ex2(x.x), p1 = ex2(x.y);
+            if (!full) {
+              p0 = key < kend ? p0 : 0.f;
+              p1 = key + 1 < kend ? p1 : 0.f;
+            }
+            ls4[(t >> 1) & 3] = fadd2(ls4[(t >> 1) & 3], f2pk(p0, p1));
             pk[t >> 1] = pack2<kBF16>(p0, p1);
           }
           tmem_st16(tbase + lane_off + kP + bj * 64 + half * 32 + c * 16, pk);
         }
+        const float2 la = f2upk(fadd2(fadd2(ls4[0], ls4[1]), fadd2(ls4[2], ls4[3])));
+        const float lsum = la.x + la.y;
         tmem_st_wait();
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) {
-          mbar_arrive(&s_free[bj]);   // S(j) consumed: its buffer may take QK(j+2)
-          mbar_arrive(&p_full[bj]);
-        }
+        if (lane == 0) mbar_arrive(&p_full[bj]);
         lpart = lpart * alpha + lsum;
-        m = m_new;
-        // O += P(j) V(j), rescaled (this thread's half of the O columns)
-        mbar_wait_warp(o_full, j & 1);
-        tc_fence_after();
-#pragma unroll
-        for (int c = 0; c < C::kHalf; c += 32) {
-          if (half * C::kHalf + c < dvn) {
-            uint32_t v[32];
-            tmem_ld32(tbase + lane_off + kO + half * C::kHalf + c, v);
-            tmem_ld_wait();
-#pragma unroll
-            for (int t = 0; t < 32; ++t) o[c + t] = o[c + t] * alpha + __uint_as_float(v[t]);
-          }
-        }
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(o_free);
       }
+      mbar_wait_warp(o_full, (nkb - 1) & 1);   // the last P.V: O is final in TMEM
+      tc_fence_after();
     }
 
     // ---- epilogue: Z = O / l.  l = both halves' sums (exchanged through shared memory).  The TMEM
@@ -408,10 +438,7 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
     for (int c0 = 0; c0 < C::kHalf; c0 += 32) {
       if (ccol0 + c0 < vw) {
         float x[32];
-        if constexpr (kLong) {
-#pragma unroll
-          for (int t = 0; t < 32; ++t) x[t] = o[c0 + t];
-        } else {
+        {
           uint32_t v[32];
           tmem_ld32(tbase + lane_off + kO + ccol0 + c0, v);
           tmem_ld_wait();
@@ -481,7 +508,7 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
 template <bool kBF16, int kDK, bool kLong, int kNKB>
 et_status launch(const CUtensorMap& tm, const CUtensorMap& tz, const AParams& prm, dim3 grid, cudaStream_t stream) {
   auto kern = attn_kernel<kBF16, kDK, kLong, kNKB>;
-  const size_t smem = 1024 + (size_t)5 * Cfg<kDK>::kOpBytes + 8 * Cfg<kDK>::kStageBytes + 2048 + 256;
+  const size_t smem = attn_smem_bytes<kLong, kDK>();
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
   std::call_once(once, [&] { attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); });
