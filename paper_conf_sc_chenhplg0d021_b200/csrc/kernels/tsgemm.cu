@@ -85,12 +85,23 @@ constexpr int kMaxBChunks = 192; // tile chunks per CTA (one single-use full bar
 constexpr int kMaxRows = 256;    // tile rows per CTA (row pointers staged in smem)
 constexpr int kMaxBiasRows = 128; // tile rows per CTA of a bias epilogue (FP32 bias staged in smem)
 constexpr int kAccCol = 384;     // first accumulator column (A uses [0, Kp/2) <= 384)
-constexpr int kMmaWarps = 8;     // warps 0-7: MMA issue, one accumulator (16 TMEM columns) each
-constexpr int kEpiGroups = 4;    // warps 8-23: epilogue, 4 groups of 4 (one warp per TMEM lane quarter);
-constexpr int kEpiWarps = 16;    //   group g drains the accumulators of MMA warps 2g and 2g + 1
-constexpr int kWarpP = kMmaWarps + kEpiWarps;   // warp 24: loads (A by TMA, tiles by bulk copy), TMEM owner
-constexpr int kFillSets = kWarpP / 4;           // warps 0-23 in 6 sets of 4 move A chunks smem -> TMEM
-constexpr int kThreads = (kWarpP + 1) * 32;
+constexpr int kAcc = 8;          // accumulators (16 TMEM columns each): a round = 8 tile rows
+// Warp roles: MMA warps [0, MW) own kAcc / MW accumulators each (accumulator a holds tile rows a,
+// a + 8, a + 16, ...); epilogue warps [MW, MW + 4 EG) form EG groups of 4 (one warp per TMEM lane
+// quarter), group g draining accumulator pairs ("pair slots" j = g, g + EG, ...; pair slot j = tile
+// rows 2j, 2j + 1); warp MW + 4 EG loads (A by TMA, tiles by bulk copy) and owns TMEM.  Measured
+// on C3's FFN1 (GELU): 8 / 4 = 15.2 us, 8 MMA warps / 5 groups = 15.6 us, 4 / 6 = 17.9 us — its
+// epilogue is throughput-bound (MUFU / FMA / TMEM reads), not short of warps, so every epilogue
+// uses 8 / 4.  A pair slot's completion is signalled on its own single-use barrier (slot_full[j]):
+// with the roles configurable a group may wait on round k + 1 of a pair before round k completed,
+// which a parity wait on a per-accumulator barrier cannot tell apart.
+template <int kEpi> struct Roles {
+  static constexpr int MW = 8;
+  static constexpr int EG = 4;
+  static constexpr int EW = 4 * EG;
+  static constexpr int WP = MW + EW;
+  static constexpr int threads = (WP + 1) * 32;
+};
 
 struct SegDev {
   const int32_t* prp;       // part_row_ptr [kparts][tile_rows + 1]
@@ -136,13 +147,13 @@ struct __align__(16) Barriers {
   uint64_t xfull[kMaxKChunks];   // A load #s landed in its slot (TMA transaction bytes)
   uint64_t xfree[kMaxKChunks];   // A load #s read out of its slot (4 fill warps)
   uint64_t a_all;                // the whole A block is in TMEM (4 fill warps x nk chunks)
-  uint64_t acc_full[kMmaWarps], acc_empty[kMmaWarps];
+  uint64_t slot_full[kMaxRows / 2], acc_empty[kAcc];   // per pair slot (single use) / per accumulator
   uint64_t bfull[kMaxBChunks];
   alignas(16) int tcol[kMaxSlots][kChunkTiles + 4];   // bulk-copy destination (16-byte aligned): tile columns
   int rptr[kMaxRows + 1];        // this CTA's row pointers, relative to its first tile
   alignas(16) float bias_f[kMaxBiasRows * 16];   // this CTA's bias slice, FP32 (converted once)
   uint32_t tmem_base;
-  int rows_seen[kEpiGroups];     // per epilogue group: rows whose MMAs were observed complete (in order)
+  uint32_t pair_done[kMaxRows / 64];   // bit j: pair slot j's MMAs observed complete (its tiles are free)
   int tcoff[kMaxSlots];          // per slot: offset of the chunk's first column index in tcol[slot]
   int a_end;                     // end (relative tile index) of part A's last row
 };
@@ -164,7 +175,7 @@ template <int kEpi> struct Smem {
   static constexpr bool kLN = kEpi == kEpiLN;
   static constexpr size_t kStageWarp = kEpi == ET_EPI_F32 ? 4096 : 2048;
   static constexpr size_t kStash = (size_t)(kLnMaxRows / 2) * 16384;
-  static constexpr size_t kStage = kLN ? kStash + sizeof(LnStats) : (size_t)kEpiWarps * kStageWarp;
+  static constexpr size_t kStage = kLN ? kStash + sizeof(LnStats) : (size_t)Roles<kEpi>::EW * kStageWarp;
   static constexpr int kSlots = kLN ? 6 : (kEpi == ET_EPI_F32 ? 9 : 11);
   static constexpr size_t kRing = (size_t)kSlots * kSlotBytes;
   static constexpr size_t kBytes = 1024 + kRing + kStage + sizeof(Barriers);
@@ -200,7 +211,7 @@ __device__ __forceinline__ void gelu_erf2(float& x0, float& x1) {
 constexpr bool is_partial(int e) { return e == ET_EPI_F32 || e == ET_EPI_PART16; }
 
 template <int kEpi, bool kBF16>
-__global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
+__global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
                                                              const __grid_constant__ CUtensorMap tmap_y,
                                                              const __grid_constant__ Params p) {
   extern __shared__ uint8_t smem_raw[];
@@ -214,6 +225,9 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   Barriers& bar = *reinterpret_cast<Barriers*>(smem + SM::kRing + SM::kStage);
 
   constexpr bool kLN = kEpi == kEpiLN;
+  constexpr int kMmaWarps = Roles<kEpi>::MW, kEpiGroups = Roles<kEpi>::EG, kEpiWarps = Roles<kEpi>::EW;
+  constexpr int kWarpP = Roles<kEpi>::WP, kFillSets = kWarpP / 4, kThreads = Roles<kEpi>::threads;
+  constexpr int kAPW = kAcc / kMmaWarps;   // accumulators per MMA warp
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const Piece pc = p.piece[blockIdx.x];
@@ -231,7 +245,8 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   const int nchA = (peA - pbA + kChunkTiles - 1) / kChunkTiles;   // part B starts on a fresh tile chunk
   const int nchunks = nchA + (peB - pbB + kChunkTiles - 1) / kChunkTiles;
   const int nrows = rowsA + rowsB;
-  const int nrounds = (nrows + kMmaWarps - 1) / kMmaWarps;   // row t is handled by MMA warp t % 8 in round t / 8
+  const int nrounds = (nrows + kAcc - 1) / kAcc;   // row t: accumulator t % 8, round t / 8
+  const int npairs_all = (nrows + 1) / 2;          // pair slots
 
   if (nchunks > kMaxBChunks || nrows > kMaxRows || (!is_partial(kEpi) && nrows > kMaxBiasRows))
     __trap();   // host sizes pieces so this cannot happen
@@ -261,12 +276,10 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       mbar_init(&bar.xfree[i], 4);
     }
     mbar_init(&bar.a_all, 4 * nk);
-    for (int i = 0; i < kMmaWarps; ++i) {
-      mbar_init(&bar.acc_full[i], 1);
-      mbar_init(&bar.acc_empty[i], 4);
-    }
+    for (int i = 0; i < kAcc; ++i) mbar_init(&bar.acc_empty[i], 4);
+    for (int j = 0; j < npairs_all; ++j) mbar_init(&bar.slot_full[j], min(2, nrows - 2 * j));   // one commit per row
     for (int i = 0; i < nchunks; ++i) mbar_init(&bar.bfull[i], 1);
-    for (int g = 0; g < kEpiGroups; ++g) bar.rows_seen[g] = 0;
+    for (int i = 0; i < kMaxRows / 64; ++i) bar.pair_done[i] = 0u;
     fence_mbar_init();
   }
   if (warp == kWarpP) tmem_alloc<512>(&bar.tmem_base);
@@ -330,6 +343,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       if (p.ts != nullptr) atomicMin(p.ts, globaltimer_ns());   // trace: this CTA's work starts
       const int kx0 = z * p.Kp;
       int tl = 0;   // last local row that starts before the end of the tile chunk being recycled
+      int pdone = 0;   // pair slots [0, pdone) known complete
       const int nseq = nk + nchunks;
       for (int s = 0; s < nseq; ++s) {
         const int slot = s % kSlots;
@@ -340,11 +354,10 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           } else {
             const int end_rel = (prev - nk + 1) * kChunkTiles;
             while (tl + 1 < nrows && bar.rptr[tl + 1] < end_rel) ++tl;
-            const int full = (tl + 1) / kMmaWarps, rem = (tl + 1) % kMmaWarps;
-#pragma unroll
-            for (int g = 0; g < kEpiGroups; ++g) {
-              const int need = 2 * full + min(max(rem - 2 * g, 0), 2);
-              while (ld_acquire_shared(&bar.rows_seen[g]) < need) {}   // (a __nanosleep back-off made every GEMM slower)
+            // pair slots 0 .. tl / 2 (rows 0 .. tl) observed complete
+            while (pdone <= (tl >> 1)) {
+              while (!((ld_acquire_shared_u32(&bar.pair_done[pdone >> 5]) >> (pdone & 31)) & 1u)) {}
+              ++pdone;
             }
           }
         }
@@ -373,7 +386,6 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
   } else if (warp < kMmaWarps) {
     // ===================== MMA warps: warp w issues the chains of tile rows w, w+8, w+16, ...
     const uint32_t idesc = make_idesc_f16(128, 16, kBF16 ? 1 : 0, 0, 0);
-    const uint32_t d_tmem = tbase + kAccCol + warp * 16;
     const uint32_t ring_u32 = smem_u32(ring);
     const int kbase = z * 48;   // first tile column of this K part
     int cur_chunk = -1;         // tile chunk whose full barrier was last waited
@@ -381,9 +393,12 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     // of this warp's issue: per-chunk waits made the first round 2-3x slower than the others)
     mbar_wait_warp(&bar.a_all, 0);
     tc_fence_after();
-    for (int k = 0; k < nrounds; ++k) {
-      const int t = k * kMmaWarps + warp;
+    for (int kk = 0; kk < nrounds * kAPW; ++kk) {
+      const int k = kk / kAPW;                     // round
+      const int acc = warp + (kk % kAPW) * kMmaWarps;   // accumulator (rows in increasing order)
+      const int t = k * kAcc + acc;
       if (t >= nrows) break;
+      const uint32_t d_tmem = tbase + kAccCol + acc * 16;
       const int q0 = bar.rptr[t], q1 = rend(t);   // this row's tiles, relative to the CTA's stream
       // The row's tiles lie in chunks [q0 / 32, (q1 - 1) / 32].  A segment = the row's tiles inside
       // one chunk: wait for the chunk once, read the tile columns lane-parallel, issue the MMAs from
@@ -413,7 +428,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
       };
       if (qb < q1) prep();
       if (k > 0) {   // the epilogue group must have read this accumulator's previous row
-        mbar_wait_warp(&bar.acc_empty[warp], (k - 1) & 1);
+        mbar_wait_warp(&bar.acc_empty[acc], (k - 1) & 1);
         tc_fence_after();
       }
       if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k);
@@ -433,7 +448,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
         qb = qe;
         if (qb < q1) prep();
       }
-      mma_commit_warp(&bar.acc_full[warp]);   // fires when this row's MMAs are complete
+      mma_commit_warp(&bar.slot_full[t >> 1]);   // fires when this row's MMAs are complete
       if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k + 2);
     }
   } else {
@@ -464,9 +479,9 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
     // one TMEM load, release them to the MMA warps, THEN do the bias / activation / store math (so
     // an MMA warp never waits for another row's epilogue arithmetic).
     float ln_n = 0.f, ln_mean = 0.f, ln_m2 = 0.f;   // kLN: running (n, mean, M2) of this thread's values
-    for (int k = 0; k < nrounds; ++k) {
-      const int t0 = k * kMmaWarps + g * 2;   // first row of this group's pair in round k
-      if (t0 >= nrows) break;
+    for (int jp = g, it = 0; jp < npairs_all; jp += kEpiGroups, ++it) {
+      const int k = jp >> 2, pidx = jp & 3;   // round, pair within the round (accumulators 2p, 2p+1)
+      const int t0 = 2 * jp;                  // first row of the pair
       const int na = min(2, nrows - t0);
       uint32_t r[32];
       uint4 res4[4];
@@ -477,18 +492,19 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
 #pragma unroll
         for (int ch = 0; ch < 4; ++ch) res4[ch] = __ldg(rp4 + ch);
       }
-      for (int a = 0; a < na; ++a) mbar_wait_warp(&bar.acc_full[g * 2 + a], k & 1);
-      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k);
+      (void)k;
+      mbar_wait_warp(&bar.slot_full[jp], 0);   // single-use: both rows' MMAs complete
+      if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it);
       tc_fence_after();
-      if (quarter == 0 && lane == 0)
-        st_release_shared(&bar.rows_seen[g], k * 2 + na);   // rows' MMAs complete: their tiles are free
-      tmem_ld32(tbase + kAccCol + g * 32 + ((uint32_t)(quarter * 32) << 16), r);
+      if (quarter == 0 && lane == 0)   // the pair's MMAs are complete: their tiles are free
+        atom_or_release_shared(&bar.pair_done[jp >> 5], 1u << (jp & 31));
+      tmem_ld32(tbase + kAccCol + pidx * 32 + ((uint32_t)(quarter * 32) << 16), r);
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
       if (lane == 0)
-        for (int a = 0; a < na; ++a) mbar_arrive(&bar.acc_empty[g * 2 + a]);
-      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 1);
+        for (int a = 0; a < na; ++a) mbar_arrive(&bar.acc_empty[pidx * 2 + a]);
+      if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it + 1);
       // math: bias / scale / activation on the pair's 32 columns of this thread's token row
       float v[32];
 #pragma unroll
@@ -530,7 +546,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           v[a * 16 + c + 1] = x1;
         }
       }
-      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 2);
+      if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it + 2);
       if constexpr (kLN) {
         // + residual; the pair's (mean, M2) merged into this thread's running statistics (Chan et
         // al.'s pairwise update); the FP32 pre-LN values go to the stash until the cluster's row
@@ -616,7 +632,7 @@ __global__ void __launch_bounds__(kThreads, 1) tsgemm_kernel(const __grid_consta
           }
         }
       }
-      if (quarter == 0 && lane == 0 && k < 8) ET_TL(208 + 40 * g + 5 * k + 3);
+      if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it + 3);
     }
     if constexpr (kLN) {
       // ===== fused residual + LayerNorm (biased variance, reading C-11).  The
@@ -751,9 +767,9 @@ et_status launch_typed(const CUtensorMap& tm, const CUtensorMap& tmy, const Para
   });
   ET_CUDA(attr_err);
   if (cluster_x > 0)
-    ET_CUDA(launch_pdl_cluster(kern, grid, dim3(kThreads), Smem<kEpi>::kBytes, stream, cluster_x, tm, tmy, prm));
+    ET_CUDA(launch_pdl_cluster(kern, grid, dim3(Roles<kEpi>::threads), Smem<kEpi>::kBytes, stream, cluster_x, tm, tmy, prm));
   else
-    ET_CUDA(launch_pdl(kern, grid, dim3(kThreads), Smem<kEpi>::kBytes, stream, tm, tmy, prm));
+    ET_CUDA(launch_pdl(kern, grid, dim3(Roles<kEpi>::threads), Smem<kEpi>::kBytes, stream, tm, tmy, prm));
   count_launch();
   return ET_OK;
 }

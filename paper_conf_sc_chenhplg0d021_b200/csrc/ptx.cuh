@@ -92,6 +92,14 @@ __device__ __forceinline__ int ld_acquire_shared(const int* p) {
   asm volatile("ld.acquire.cta.shared::cta.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
   return v;
 }
+__device__ __forceinline__ uint32_t ld_acquire_shared_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.cta.shared::cta.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ void atom_or_release_shared(uint32_t* p, uint32_t bits) {
+  asm volatile("red.release.cta.shared::cta.or.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(bits) : "memory");
+}
 __device__ __forceinline__ void st_release_shared(int* p, int v) {
   asm volatile("st.release.cta.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
