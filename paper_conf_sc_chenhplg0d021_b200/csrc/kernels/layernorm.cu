@@ -264,7 +264,7 @@ __device__ __forceinline__ void layernorm_row8(const LnArgs& a) {
 }
 
 template <int NCH, int NP, int DT, int RT, bool P16>
-__global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
+__global__ void __launch_bounds__(512) layernorm_kernel(const LnArgs a) {
   pdl_trigger();
   pdl_wait();
   trace_cta_start(a.ts);
@@ -278,7 +278,9 @@ __global__ void __launch_bounds__(128) layernorm_kernel(const LnArgs a) {
 
 template <int NCH, int DT, int RT, bool P16>
 et_status launch_np(const LnArgs& a, cudaStream_t stream) {
-  const int threads = 128;
+  // rows per CTA (one warp each): ET_LN_THREADS (experiment knob; default 128 threads = 4 rows)
+  static const int env_threads = getenv("ET_LN_THREADS") ? atoi(getenv("ET_LN_THREADS")) : 128;
+  const int threads = (env_threads == 256 || env_threads == 512) ? env_threads : 128;
   const int blocks = (a.M * 32 + threads - 1) / threads;
   cudaError_t e = cudaSuccess;
   switch (a.nparts) {
