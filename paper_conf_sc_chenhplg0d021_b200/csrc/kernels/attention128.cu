@@ -141,20 +141,33 @@ __global__ void __launch_bounds__(kThreads, 3) attn128_kernel(const __grid_const
     const float sl2 = p.scale_log2;
     mbar_wait_warp(s_full, 0);
     tc_fence_after();
-    // pass 1: row maximum over the valid keys
-    float m = -INFINITY;
+    // pass 1: row maximum over the valid keys (8 independent partial maxima: no 128-long chain;
+    // rows with every key valid skip the per-key predicate)
+    const bool full = kend >= 128;
+    float mx8[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) mx8[i] = -INFINITY;
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
       uint32_t v[32];
       tmem_ld32(tbase + lane_off + c * 32, v);
       tmem_ld_wait();
+      if (full) {
 #pragma unroll
-      for (int t = 0; t < 32; ++t)
-        if (c * 32 + t < kend) m = fmaxf(m, __uint_as_float(v[t]));
+        for (int t = 0; t < 32; ++t) mx8[t & 7] = fmaxf(mx8[t & 7], __uint_as_float(v[t]));
+      } else {
+#pragma unroll
+        for (int t = 0; t < 32; ++t)
+          if (c * 32 + t < kend) mx8[t & 7] = fmaxf(mx8[t & 7], __uint_as_float(v[t]));
+      }
     }
+    const float m = fmaxf(fmaxf(fmaxf(mx8[0], mx8[1]), fmaxf(mx8[2], mx8[3])),
+                          fmaxf(fmaxf(mx8[4], mx8[5]), fmaxf(mx8[6], mx8[7])));
     const float mb = m * sl2;
-    // pass 2: p = 2^(s log2e - m log2e) (exactly 0 for masked keys), row sum, P in place
-    float l = 0.f;
+    // pass 2: p = 2^(s log2e - m log2e) (exactly 0 for masked keys), row sum (4 packed partial
+    // sums), P in place; the exponent arguments two at a time (FFMA2)
+    uint64_t ls4[4] = {0ull, 0ull, 0ull, 0ull};
+    const uint64_t sl2x2 = f2pk(sl2, sl2), nmb2 = f2pk(-mb, -mb);
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
       uint32_t v[32];
@@ -163,13 +176,19 @@ __global__ void __launch_bounds__(kThreads, 3) attn128_kernel(const __grid_const
       uint32_t pk[16];
 #pragma unroll
       for (int t = 0; t < 32; t += 2) {
-        const float p0 = c * 32 + t < kend ? ex2f(__uint_as_float(v[t]) * sl2 - mb) : 0.f;
-        const float p1 = c * 32 + t + 1 < kend ? ex2f(__uint_as_float(v[t + 1]) * sl2 - mb) : 0.f;
-        l += p0 + p1;
+        const float2 x = f2upk(ffma2(f2pk(__uint_as_float(v[t]), __uint_as_float(v[t + 1])), sl2x2, nmb2));
+        float p0 = ex2f(x.x), p1 = ex2f(x.y);
+        if (!full) {
+          p0 = c * 32 + t < kend ? p0 : 0.f;
+          p1 = c * 32 + t + 1 < kend ? p1 : 0.f;
+        }
+        ls4[(t >> 1) & 3] = fadd2(ls4[(t >> 1) & 3], f2pk(p0, p1));
         pk[t >> 1] = pack2<kBF16>(p0, p1);
       }
       tmem_st16(tbase + lane_off + c * 16, pk);
     }
+    const float2 la = f2upk(fadd2(fadd2(ls4[0], ls4[1]), fadd2(ls4[2], ls4[3])));
+    const float l = la.x + la.y;
     tmem_st_wait();
     tc_fence_before();
     __syncwarp();
