@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--config", default="C3")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-parity", action="store_true", help="skip the sampled oracle comparison in the line")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the cpu_baseline sample")
     ap.add_argument("--parallel", choices=["batch", "head"], default="batch",
                     help="batch: batch sharding (default, weak scaling); head: head-parallel latency mode "
@@ -230,6 +231,40 @@ def oracle_seqs_per_s(cfg, raws, X, lens, budget_s: float, chunk: int):
         el = time.perf_counter() - t0
         if el >= budget_s:
             return done / el, done, el
+
+
+def parity_sample(cfg, raws, X, lens, Y, layers_packed, nseq: int = 2):
+    """SURVEY §8(d) line fields: the GPU output of the first `nseq` sequences of the timed batch
+    against the float64 oracle (max-abs, relative Frobenius), and layer 0's six packed masks against
+    the oracle's selection (bit-exact).  Test infrastructure only: it runs after the timed regions."""
+    from oracle import encoder as oe
+    pruned = [oe.prune_layer(r, cfg.scheme, cfg.ratio) for r in raws]
+    ref = oe.encoder(X[:nseq].astype(np.float64), [p[0] for p in pruned], cfg.heads, lens[:nseq], cfg.causal,
+                     cfg.act, cfg.ln_eps).reshape(nseq * cfg.seq_len, cfg.d_model)
+    got = Y[: nseq * cfg.seq_len].float().cpu().numpy().astype(np.float64)
+    d = got - ref
+    masks_ok = True
+    for n in ("wq", "wk", "wv", "wo", "w1", "w2"):
+        want = pruned[0][1][n]["mask"]
+        have = layers_packed[0].packed[n].mask().cpu().numpy().view(np.uint32)[: want.size]
+        masks_ok = masks_ok and bool(np.array_equal(have, want))
+    return {"sequences": nseq, "max_abs": float(np.abs(d).max()),
+            "rel_fro": float(np.linalg.norm(d) / np.linalg.norm(ref)), "tol_max_abs": 2e-2, "tol_rel_fro": 5e-3,
+            "masks_bit_exact_layer0": masks_ok}
+
+
+def git_sha():
+    """The revision libet.so was built from (build/BUILD_SHA, written by build.py), else git."""
+    try:
+        with open(os.path.join(ROOT, "build", "BUILD_SHA")) as fh:
+            return fh.read().strip() or None
+    except OSError:
+        pass
+    try:
+        return subprocess.run(["git", "rev-parse", "--short", "HEAD"], cwd=ROOT, capture_output=True, text=True,
+                              timeout=5).stdout.strip() or None
+    except Exception:
+        return None
 
 
 def cpu_threads():
@@ -443,6 +478,9 @@ def our_arm(args):
                         "peak_src": pk["src"] + " hbm_gbs"}
         share = {k: round(v / sum(tot.values()), 4) for k, v in tot.items()} if tot else {}
         kern_ms = {k: round(statistics.mean(v), 5) for k, v in per_kind.items()}
+        # stepwise roofline: sum over the layer's kernels of max(F/P_tc, B/P_hbm)
+        t_roof = cfg.layers * sum(max(f / (pk["bf16_tflops_sustained"] * 1e12), b / (pk["hbm_gbs"] * 1e9))
+                                  for b, f in model.values() if (b, f) != (0, 0))
         eflops = eff_flops_per_step(cfg, nnz_layers) * world
         ns = {"eff_tflops": eflops * K / t_max / 1e12}
         ns["frac_of_measured_tc"] = ns["eff_tflops"] / pk["bf16_tflops"]
@@ -462,12 +500,17 @@ def our_arm(args):
             "gpu_launches": int(launches),
             "clocks": clocks,
             "step_ms_p50": statistics.median(step_ms),
+            "step_ms_p10": float(np.percentile(step_ms, 10)), "step_ms_p90": float(np.percentile(step_ms, 90)),
+            "stepwise_roofline_frac": t_roof / (t_max / K),
+            "git": git_sha(),
             "traced_step_ms_p50": statistics.median(tr_ms),
             "launch": "one CUDA graph replay per step (et_encoder_graph_create / et_graph_launch)",
         }
         if e2e:
             line["e2e"] = {"value": total_seqs / e2e_max, "unit": "seqs/s", "h2d_bytes_per_step": e2e["h2d"],
                            "d2h_bytes_per_step": e2e["d2h"]}
+        if not args.no_parity:
+            line["parity"] = parity_sample(cfg, raws, X, lens, out, layers)
         if world == 1 and not args.no_cpu_baseline:
             v, n, el = oracle_seqs_per_s(cfg, raws, X, lens, args.cpu_seconds, chunk=2)
             line["cpu_baseline"] = {"value": v, "unit": "seqs/s", "cores": cpu_threads(), "kind": "oracle",

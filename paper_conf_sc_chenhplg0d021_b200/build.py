@@ -83,6 +83,17 @@ def build(verbose: bool = False, force: bool = False, debug: bool = False, varia
         run([nvcc, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-ldl",
              "-lrt", "-lpthread"])
         os.replace(tmp, lib)
+    # the source revision the library was built from (bench.py reports it; the GPU box has no .git)
+    try:
+        sha = subprocess.run(["git", "rev-parse", "--short", "HEAD"], cwd=ROOT, capture_output=True, text=True,
+                             timeout=5).stdout.strip()
+        dirty = subprocess.run(["git", "status", "--porcelain", "--untracked-files=no"], cwd=ROOT,
+                               capture_output=True, text=True, timeout=5).stdout.strip()
+        if sha:
+            with open(os.path.join(ROOT, "build", "BUILD_SHA"), "w") as fh:
+                fh.write(sha + ("-dirty" if dirty else "") + "\n")
+    except Exception:
+        pass
     return lib
 
 
