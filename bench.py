@@ -238,6 +238,7 @@ def parity_sample(cfg, raws, X, lens, Y, layers_packed, nseq: int = 2):
     against the float64 oracle (max-abs, relative Frobenius), and layer 0's six packed masks against
     the oracle's selection (bit-exact).  Test infrastructure only: it runs after the timed regions."""
     from oracle import encoder as oe
+    nseq = min(nseq, cfg.batch)
     pruned = [oe.prune_layer(r, cfg.scheme, cfg.ratio) for r in raws]
     ref = oe.encoder(X[:nseq].astype(np.float64), [p[0] for p in pruned], cfg.heads, lens[:nseq], cfg.causal,
                      cfg.act, cfg.ln_eps).reshape(nseq * cfg.seq_len, cfg.d_model)
