@@ -133,6 +133,19 @@ et_status et_prune_pack(const void* W_dev, int32_t rows, int32_t cols, et_dtype 
  * to check values bit-exactly).  dense_out: device [rows, cols] in the packed dtype. */
 et_status et_unpack(const et_packed_weight* w, void* dense_out, void* stream);
 
+/* Column gather for column pruning with X_adjusted (§4.1, Fig. 5(b)):
+ *   out[r, j] = in[r * ld_in + idx[j]]   for j < nk;   out[r, j] = 0 for nk <= j < nk_pad
+ * The column-pruned linear layer is X_adjusted . W_pruned^T: gather the kept columns of W once
+ * (W_pruned = condensed [rows, nk_pad] weight, then packed as a dense tile weight with ratio 0) and
+ * the kept columns of X per call (X_adjusted [M, nk_pad]); padded columns are zero on both sides,
+ * so the product is exact.  idx_dev: device int32 [nk], the kept column indices (out->idx of an
+ * ET_PRUNE_COL et_prune_pack, ascending).  in: device [rows, ld_in]; out: device [rows, nk_pad],
+ * 16-byte aligned; dtype FP16/BF16 (bits moved as-is) or FP32.  nk_pad % 8 == 0 (FP32: % 4 == 0)
+ * else ET_ERR_INVALID_ARG; idx values outside [0, ld_in) are undefined behaviour.  Stream-ordered,
+ * graph capturable, no allocation. */
+et_status et_gather_cols(const void* in, int32_t rows, int32_t ld_in, const int32_t* idx_dev, int32_t nk,
+                         int32_t nk_pad, et_dtype dtype, void* out, void* stream);
+
 /* ------------------------------------------------------------------------------------------
  * Tile-sparse linear layer (test hook + building block):
  *   Y[M, N] = epilogue(X[M, K] . W'^T + b)         N = w->rows (ROW: rows_padded), K = w->cols

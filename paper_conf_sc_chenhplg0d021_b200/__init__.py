@@ -227,6 +227,44 @@ def linear_fwd(w: Packed, X: torch.Tensor, bias: torch.Tensor | None = None, epi
     return out
 
 
+_gather = _sig("et_gather_cols", ctypes.c_int, [_vp, _i32, _i32, _vp, _i32, _i32, ctypes.c_int, _vp, _vp])
+SYMBOLS += ["et_gather_cols"]
+
+
+def gather_cols(A: torch.Tensor, idx: torch.Tensor, nk_pad: int, out: torch.Tensor | None = None, stream=None):
+    """et_gather_cols: out[r, j] = A[r, idx[j]] (j < len(idx)), 0 up to nk_pad (X_adjusted)."""
+    assert A.is_cuda and A.dim() == 2 and A.is_contiguous() and idx.dtype == torch.int32
+    if out is None:
+        out = torch.empty(A.shape[0], nk_pad, dtype=A.dtype, device=A.device)
+    _check(_gather(A.data_ptr(), A.shape[0], A.shape[1], _ptr(idx) if idx.numel() else None, idx.numel(), nk_pad,
+                   dtype_code(A.dtype), out.data_ptr(), _stream(stream)))
+    return out
+
+
+class ColLinear:
+    """Column-pruned linear layer with X_adjusted (Fig. 5(b)).
+
+    pack: et_prune_pack(ET_PRUNE_COL) selects the kept input columns (mask / ascending idx, bit-exact
+    with the oracle); W_pruned = W[:, keep] is condensed by et_gather_cols, zero-padded to a multiple
+    of 64 columns (the tile GEMM's K granule) and packed as a dense tile weight (ratio 0).
+    forward: X_adjusted = et_gather_cols(X, keep) (one gather kernel), then the tcgen05 tile GEMM
+    (et_linear_fwd) on the condensed operands.  Padded columns are zero on both sides (exact)."""
+
+    def __init__(self, W: torch.Tensor, ratio: float, stream=None):
+        self.rows, self.cols = W.shape
+        self.sel = prune_pack(W, "col", ratio, stream=stream)
+        self.nk = self.sel.nnz
+        self.keep = self.sel.kept_index()
+        self.nk_pad = max(64, (self.nk + 63) // 64 * 64)
+        Wc = gather_cols(W, self.keep, self.nk_pad, stream=stream)
+        self.dense = prune_pack(Wc, "tile", 0.0, stream=stream)
+
+    def __call__(self, X: torch.Tensor, bias: torch.Tensor | None = None, epi: int = EPI_BIAS, stream=None,
+                 x_adj: torch.Tensor | None = None):
+        Xa = gather_cols(X, self.keep, self.nk_pad, out=x_adj, stream=stream)
+        return linear_fwd(self.dense, Xa, bias, epi, stream=stream)
+
+
 def layernorm_fwd(part: torch.Tensor, bias, resid, gamma, beta, eps: float, dtype, resid_dtype,
                   out_act=None, out_resid=None, stream=None):
     """et_layernorm_fwd: LN(sum(part) + bias + resid)."""

@@ -195,6 +195,18 @@ et_status et_unpack(const et_packed_weight* w, void* dense_out, void* stream) {
   return unpack_run(w, dense_out, static_cast<cudaStream_t>(stream));
 }
 
+et_status et_gather_cols(const void* in, int32_t rows, int32_t ld_in, const int32_t* idx_dev, int32_t nk,
+                         int32_t nk_pad, et_dtype dtype, void* out, void* stream) {
+  if (rows < 0 || nk < 0 || nk_pad < nk || ld_in < 0) return fail(ET_ERR_INVALID_ARG, "et_gather_cols: bad sizes");
+  if (!valid_dtype(dtype)) return fail(ET_ERR_INVALID_ARG, "et_gather_cols: bad dtype");
+  const int V = dtype == ET_FP32 ? 4 : 8;
+  if (nk_pad % V) return fail(ET_ERR_INVALID_ARG, "et_gather_cols: nk_pad must be a multiple of %d", V);
+  if (rows == 0 || nk_pad == 0) return ET_OK;
+  if (!in || !out || (nk > 0 && !idx_dev)) return fail(ET_ERR_INVALID_ARG, "et_gather_cols: null pointer");
+  if (!aligned16(out)) return fail(ET_ERR_INVALID_ARG, "et_gather_cols: out not 16B aligned");
+  return gather_cols_run(in, rows, ld_in, idx_dev, nk, nk_pad, dtype, out, static_cast<cudaStream_t>(stream));
+}
+
 static et_status segment_from(const et_packed_weight* w, const void* bias, GemmSegment* sg, int out_col) {
   if (!w->values || !w->part_row_ptr || !w->tile_col)
     return fail(ET_ERR_INVALID_ARG, "packed weight has no values / part_row_ptr / tile_col");

@@ -148,6 +148,10 @@ struct VPrep {
 };
 et_status vprep_run(const VPrep& v, cudaStream_t stream);
 
+// column pruning (kernels/colgather.cu): Out[r, j] = In[r, idx[j]] (j < nk), 0 for nk <= j < nk_pad
+et_status gather_cols_run(const void* in, int rows, int ld_in, const int32_t* idx, int nk, int nk_pad, et_dtype dt,
+                          void* out, cudaStream_t stream);
+
 // ---------------------------------------------------------------- tracing (api.cu)
 // Record a mark of `kind` on `stream` if tracing is enabled; counts one kernel launch.
 unsigned long long* trace_slot(int kind);

@@ -64,6 +64,18 @@ def test_prune_pack_query_rejects_bad_arguments(et):
     assert _query(et, 768, 768, et.FP16, et.PRUNE_ROW, 0.5, group=100)[0] == 1
 
 
+def test_gather_cols_validates_before_launch(et):
+    # et_gather_cols (column pruning, X_adjusted): argument errors return before any
+    # CUDA call, so they are checkable on a CPU-only host
+    g = et._gather
+    assert g(None, 4, 64, None, 10, 12, et.FP16, None, None) == 1          # nk_pad % 8 != 0
+    assert "multiple" in et._lib.et_last_error().decode()
+    assert g(None, 4, 64, None, 10, 8, et.FP16, None, None) == 1           # nk_pad < nk
+    assert g(None, 4, 64, None, 4, 8, 7, None, None) == 1                  # bad dtype
+    assert g(None, 4, 64, None, 4, 8, et.FP16, None, None) == 1            # null pointers
+    assert g(None, 0, 64, None, 0, 8, et.FP16, None, None) == 0            # empty: nothing to do
+
+
 def test_product_has_no_cpu_fallback(et):
     import torch
     if torch.cuda.is_available():

@@ -22,17 +22,34 @@ except Exception:
     pass
 
 
-def timed(fn, reps=50, warm=5):
+def timed(fn, reps=50, warm=5, graph=True):
+    """Device time per call (us).  graph=True: `reps` calls captured in one CUDA graph and the graph
+    replayed, so host launch overhead (ctypes + torch, several us per call) is not measured."""
     for _ in range(warm):
         fn()
     torch.cuda.synchronize()
+    if graph:
+        g = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            with torch.cuda.graph(g, stream=s):
+                for _ in range(reps):
+                    fn()
+        torch.cuda.current_stream().wait_stream(s)
+        g.replay()
+        torch.cuda.synchronize()
+        run = g.replay
+        n = reps
+    else:
+        run = lambda: [fn() for _ in range(reps)]
+        n = reps
     a, b = torch.cuda.Event(True), torch.cuda.Event(True)
     a.record()
-    for _ in range(reps):
-        fn()
+    run()
     b.record()
     torch.cuda.synchronize()
-    return a.elapsed_time(b) / reps * 1e3   # us
+    return a.elapsed_time(b) / n * 1e3   # us
 
 
 def m2():
@@ -58,6 +75,36 @@ def m2():
                               "dense_torch_matmul_us": round(dense_us, 2)}), flush=True)
 
 
+def m2b():
+    """Pruning-method comparison (Fig. 10 / line 252 analogue): tile vs row vs column
+    pruned linear layer, d x d at M = 4096 tokens (S = 128, B = 32), ratio 0 ... 0.95.  Row: condensed
+    output rows (padded to 16); column: X_adjusted gather + condensed-K tile GEMM (both launches
+    timed)."""
+    M = 4096
+    for d in (768, 1024):
+        W = torch.tensor(make_matrix(5, (d, d), 0.02, "fp16"), dtype=torch.float16, device="cuda")
+        X = torch.tensor(make_matrix(6, (M, d), 1.0, "fp16"), dtype=torch.float16, device="cuda")
+        dense_us = timed(lambda: torch.matmul(X, W.t()))
+        for ratio in (0.0, 0.2, 0.4, 0.6, 0.8, 0.9, 0.95):
+            row = {"sweep": "M2b", "d": d, "M": M, "ratio": ratio, "dense_torch_matmul_us": round(dense_us, 2)}
+            epi = et.EPI_PART16 if d > 768 else et.EPI_BIAS
+            pk = et.prune_pack(W, "tile", ratio)
+            out = et.linear_fwd(pk, X, None, epi)
+            row["tile_us"] = round(timed(lambda: et.linear_fwd(pk, X, None, epi, out=out)), 2)
+            pr = et.prune_pack(W, "row", ratio)
+            out_r = et.linear_fwd(pr, X, None, epi)
+            row["row_us"] = round(timed(lambda: et.linear_fwd(pr, X, None, epi, out=out_r)), 2)
+            cl = et.ColLinear(W, ratio)
+            xa = torch.empty(M, cl.nk_pad, dtype=X.dtype, device="cuda")
+            epi_c = et.EPI_PART16 if cl.nk_pad > 768 else et.EPI_BIAS
+            out_c = et.linear_fwd(cl.dense, xa, None, epi_c)
+            row["col_gather_us"] = round(timed(lambda: et.gather_cols(X, cl.keep, cl.nk_pad, out=xa)), 2)
+            row["col_gemm_us"] = round(timed(lambda: et.linear_fwd(cl.dense, xa, None, epi_c, out=out_c)), 2)
+            row["col_us"] = round(row["col_gather_us"] + row["col_gemm_us"], 2)
+            row["col_kept"] = cl.nk
+            print(json.dumps(row), flush=True)
+
+
 def m3():
     H, dk, total = 12, 64, 32768
     d = H * dk
@@ -77,8 +124,10 @@ def m3():
 
 
 if __name__ == "__main__":
-    which = sys.argv[1:] or ["m2", "m3"]
+    which = sys.argv[1:] or ["m2", "m2b", "m3"]
     if "m2" in which:
         m2()
+    if "m2b" in which:
+        m2b()
     if "m3" in which:
         m3()
