@@ -32,21 +32,31 @@ __global__ void cast_kernel(const void* __restrict__ src, et_dtype sdt, void* __
   for (size_t i = i0; i < n && i < i0 + 4; ++i) stf(dst, ddt, i, ldf(src, sdt, i));
 }
 
-// single thread: per-head segments of the packed (padded) V rows
-__global__ void vprep_heads_kernel(const int32_t* __restrict__ idx, int nnz, int heads, int d_k,
+// per-head segments of the packed (padded) V rows: thread h counts head h's kept rows from the row
+// bitmap (popcount over bits [h d_k, (h+1) d_k)), pads it to 16, and sums the padded widths of the
+// heads before it.  No serial pointer chase (a single-thread walk over idx cost one dependent global
+// load per kept row, ~30 us per forward on C2).
+__global__ void vprep_heads_kernel(const uint32_t* __restrict__ mask, int heads, int d_k,
                                    int32_t* __restrict__ v_col, int32_t* __restrict__ v_width) {
-  if (threadIdx.x || blockIdx.x) return;
-  int k = 0, start = 0;
-  for (int h = 0; h < heads; ++h) {
+  extern __shared__ int32_t s_pad[];
+  for (int h = threadIdx.x; h < heads; h += blockDim.x) {
+    const int b0 = h * d_k, b1 = b0 + d_k;
     int cnt = 0;
-    while (k < nnz && idx[k] / d_k == h) {
-      ++cnt;
-      ++k;
+    for (int w = b0 >> 5; w <= (b1 - 1) >> 5; ++w) {
+      uint32_t m = __ldg(mask + w);
+      const int lo = max(b0 - w * 32, 0), hi = min(b1 - w * 32, 32);   // bits [lo, hi) of word w
+      if (hi < 32) m &= (1u << hi) - 1u;
+      m &= ~((1u << lo) - 1u);
+      cnt += __popc(m);
     }
-    const int pad = (cnt + 15) / 16 * 16;
+    s_pad[h] = (cnt + 15) / 16 * 16;
+  }
+  __syncthreads();
+  for (int h = threadIdx.x; h < heads; h += blockDim.x) {
+    int start = 0;
+    for (int k = 0; k < h; ++k) start += s_pad[k];
     v_col[h] = start;
-    v_width[h] = pad;
-    start += pad;
+    v_width[h] = s_pad[h];
   }
 }
 
@@ -58,36 +68,41 @@ __global__ void vprep_bias_kernel(const int32_t* __restrict__ row_map, int rows_
   stf(bv_packed, dt, i, r >= 0 ? ldf(bv, dt, r) : 0.f);
 }
 
-// one thread per output feature i of W_O (tile pruned): walk the kept tiles of its tile row in a
-// fixed order (deterministic), add W_O'[i, f] * b_V[f] for every pruned V feature f.
+// one warp per output feature i of W_O (tile pruned): the lanes stride over the (kept tile, k) pairs of
+// its tile row (every K part), add W_O'[i, f] * b_V[f] for every pruned V feature f in FP64, and
+// combine in a fixed butterfly (deterministic).  (One thread per feature walking the row serially
+// was the longest kernel of a C2 forward: 27 us on 4 SMs.)
 __global__ void vprep_fold_kernel(const uint8_t* __restrict__ wo_values, const int32_t* __restrict__ wo_prp,
                                   const int32_t* __restrict__ wo_tile_col, int wo_tile_rows, int kparts,
                                   const uint32_t* __restrict__ wv_mask, const void* __restrict__ bv,
                                   const void* __restrict__ bo, et_dtype dt, int d, void* __restrict__ bo_folded) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
   if (i >= d) return;
   const int ti = i >> 4, n = i & 15;
   double acc = 0.0;
   for (int z = 0; z < kparts; ++z) {
     const int32_t* rp = wo_prp + z * (wo_tile_rows + 1);
-    for (int t = rp[ti]; t < rp[ti + 1]; ++t) {
-      const int j = wo_tile_col[t];
+    const int t0 = rp[ti], ne = (rp[ti + 1] - t0) * 16;
+    for (int e = lane; e < ne; e += 32) {
+      const int t = t0 + (e >> 4), k = e & 15;
+      const int f = wo_tile_col[t] * 16 + k;
+      if ((wv_mask[f >> 5] >> (f & 31)) & 1u) continue;   // kept V feature: no fold
       const uint8_t* tile = wo_values + (size_t)t * 256 * (dt == ET_FP32 ? 4 : 2);
-      for (int k = 0; k < 16; ++k) {
-        const int f = j * 16 + k;
-        if ((wv_mask[f >> 5] >> (f & 31)) & 1u) continue;   // kept V feature: no fold
-        float w;
-        if (dt == ET_FP32) {   // FP32 tiles: row-major (simt32.cu)
-          w = *reinterpret_cast<const float*>(tile + n * 64 + k * 4);
-        } else {
-          const uint16_t raw = *reinterpret_cast<const uint16_t*>(tile + (n >> 3) * 256 + (k >> 3) * 128 + (n & 7) * 16 + (k & 7) * 2);
-          w = dt == ET_BF16 ? __bfloat162float(__ushort_as_bfloat16(raw)) : __half2float(__ushort_as_half(raw));
-        }
-        acc += (double)w * (double)ldf(bv, dt, f);
+      float w;
+      if (dt == ET_FP32) {   // FP32 tiles: row-major (simt32.cu)
+        w = *reinterpret_cast<const float*>(tile + n * 64 + k * 4);
+      } else {   // 16-bit tiles: tcgen05 core-matrix layout
+        const uint16_t raw = *reinterpret_cast<const uint16_t*>(tile + (n >> 3) * 256 + (k >> 3) * 128 + (n & 7) * 16 + (k & 7) * 2);
+        w = dt == ET_BF16 ? __bfloat162float(__ushort_as_bfloat16(raw)) : __half2float(__ushort_as_half(raw));
       }
+      acc += (double)w * (double)ldf(bv, dt, f);
     }
   }
-  stf(bo_folded, dt, i, (float)((bo ? (double)ldf(bo, dt, i) : 0.0) + acc));   // bo NULL: fold only (head-parallel rank)
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (lane == 0)   // bo NULL: fold only (head-parallel rank)
+    stf(bo_folded, dt, i, (float)((bo ? (double)ldf(bo, dt, i) : 0.0) + acc));
 }
 
 }  // namespace
@@ -104,7 +119,9 @@ et_status cast_run(const void* src, et_dtype sdt, void* dst, et_dtype ddt, size_
 et_status vprep_run(const VPrep& v, cudaStream_t stream) {
   if (v.wv->pattern != ET_PRUNE_ROW) return fail(ET_ERR_INTERNAL, "vprep: W_V is not row pruned");
   if (v.wo->pattern != ET_PRUNE_TILE) return fail(ET_ERR_UNSUPPORTED, "vprep: W_O must be tile pruned");
-  vprep_heads_kernel<<<1, 32, 0, stream>>>(v.wv->idx, v.wv->nnz, v.heads, v.d_k, v.v_col, v.v_width);
+  const int ht = v.heads < 1024 ? (v.heads + 31) / 32 * 32 : 1024;
+  vprep_heads_kernel<<<1, ht, v.heads * sizeof(int32_t), stream>>>(v.wv->mask, v.heads, v.d_k, v.v_col,
+                                                                  v.v_width);
   count_launch();
   ET_CUDA(cudaGetLastError());
   if (v.wv->rows_padded > 0) {
@@ -114,7 +131,7 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream) {
     ET_CUDA(cudaGetLastError());
   }
   const int d = v.wo->rows;
-  vprep_fold_kernel<<<(d + 127) / 128, 128, 0, stream>>>(static_cast<const uint8_t*>(v.wo->values),
+  vprep_fold_kernel<<<(d + 3) / 4, 128, 0, stream>>>(static_cast<const uint8_t*>(v.wo->values),
                                                          v.wo->part_row_ptr, v.wo->tile_col, v.wo->rows / 16,
                                                          v.wo->kparts, v.wv->mask, v.bv, v.bo, v.dtype, d,
                                                          v.bo_folded);
