@@ -71,6 +71,7 @@ struct AParams {
   float scale_log2;         // scale * log2(e)
   int box_rows;             // TMA box height: min(128, total rows)
   int tma_store;            // Z written through TMA stores (dense V layout, seq_len % 32 == 0)
+  int z_stage;              // z_map scatter staged in shared memory, stored as 16-byte row windows
   unsigned long long* ts;   // trace slot or nullptr
 };
 
@@ -111,7 +112,11 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
   pdl_trigger();
   pdl_wait();   // QKV (and the attention-aware head tables) of the predecessors are visible from here
   trace_cta_start(p.ts);
-  if (p.v_width && p.v_width[p.head_begin + blockIdx.y] == 0) {   // every V feature of the head pruned
+  // attention-aware head tables: both loads issued together (one latency, not two in series)
+  const int hh = p.head_begin + blockIdx.y;
+  const int vloc = p.v_col ? __ldg(p.v_col + hh) : hh * kDK;   // packed V column of this head
+  const int vw = p.v_width ? __ldg(p.v_width + hh) : kDK;
+  if (vw == 0) {   // every V feature of the head pruned
     trace_cta_end(p.ts);
     return;
   }
@@ -148,9 +153,7 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
   const int nkb = (kmax + 127) / 128;
   const int row0 = b * S;                          // first token row of this sequence
   const int qcol = p.q_off + h * kDK, kcol = p.k_off + h * kDK;
-  const int vloc = p.v_col ? p.v_col[h] : h * kDK; // packed V column of this head
   const int vcol = p.v_off + vloc;
-  const int vw = p.v_width ? p.v_width[h] : kDK;
   const int dvn = p.dv_max;                        // P.V MMA N
 
   if (p.box_rows < 128) {
@@ -432,6 +435,19 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
     // either all valid or all beyond the sequence — those must not be written at all)
     const bool tma_warp = p.tma_store && (qb * 128 + quarter * 32 < S);
     const int ccol0 = half * C::kHalf;           // first O column of this thread
+    // attention-aware Z (z_map, row-pruned V): the head's kept columns scatter into its kDK-wide
+    // window of Z.  Staged: the window of all 128 rows is built in the (now idle) Q buffer —
+    // zero-filled, 16-byte unit u of row r at u ^ (r % 8) — then stored as whole 16-byte units by
+    // consecutive threads (a direct scatter wrote 2-byte elements, one row per lane: 32 lines per
+    // store instruction).  Every MMA has completed (O is final), so sQ is free.
+    const bool zst = p.z_map && p.z_stage;
+    const int etid = sw * 32 + lane;             // 0..255 over the softmax / epilogue warps
+    int zwb = 0;                                 // first Z column of this head's window
+    if (zst) {
+      zwb = (__ldg(p.z_map + vloc) / kDK) * kDK;  // a head's first packed V column is a kept feature
+      for (int i = etid; i < C::kOpBytes / 16; i += 256) reinterpret_cast<uint4*>(sQ)[i] = make_uint4(0, 0, 0, 0);
+      named_bar_sync(1, 256);
+    }
     uint8_t* st = sStage + sw * C::kStageBytes;  // 32 rows x kHalf fp16, 64-byte rows (SWIZZLE_64B)
     T* zrow = static_cast<T*>(p.Z) + (size_t)(row0 + qi) * p.ld_z;
 #pragma unroll
@@ -455,6 +471,19 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
                                        pack2<kBF16>(x[8 * ch + 6] * inv, x[8 * ch + 7] * inv));
             *reinterpret_cast<uint4*>(st + (c0 / 32) * 2048 + lane * 64 + ((ch ^ ((lane >> 1) & 3)) << 4)) = u;
           }
+        } else if (zst) {
+          const int32_t* zm = p.z_map + vloc + ccol0 + c0;
+#pragma unroll
+          for (int t = 0; t < 32; ++t)
+            if (ccol0 + c0 + t < vw) {
+              const int dst = __ldg(zm + t);
+              if (dst >= 0) {
+                const int j = dst - zwb;
+                T* e = reinterpret_cast<T*>(sQ + r * (kDK * 2) + (((j >> 3) ^ (r & 7)) << 4) + (j & 7) * 2);
+                if constexpr (kBF16) *e = __float2bfloat16_rn(x[t] * inv);
+                else *e = __float2half_rn(x[t] * inv);
+              }
+            }
         } else if (store && !p.tma_store) {
           if (p.z_map) {
             const int32_t* zm = p.z_map + vloc + ccol0 + c0;
@@ -477,6 +506,16 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
                     pack2<kBF16>(x[t + 4] * inv, x[t + 5] * inv), pack2<kBF16>(x[t + 6] * inv, x[t + 7] * inv));
           }
         }
+      }
+    }
+    if (zst) {
+      named_bar_sync(1, 256);
+      constexpr int kU = kDK / 8;                // 16-byte units per row window
+      for (int i = etid; i < 128 * kU; i += 256) {
+        const int r2 = i / kU, u = i % kU;
+        if (qb * 128 + r2 < S)
+          *reinterpret_cast<uint4*>(static_cast<T*>(p.Z) + (size_t)(row0 + qb * 128 + r2) * p.ld_z + zwb + u * 8) =
+              *reinterpret_cast<const uint4*>(sQ + r2 * (kDK * 2) + ((u ^ (r2 & 7)) << 4));
       }
     }
     if (tma_warp) {
@@ -556,6 +595,7 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   // TMA stores of Z: dense per-head V, every 32-row group inside one sequence, Z 16-byte aligned
   prm.tma_store = (a.z_map == nullptr && a.v_width == nullptr && a.seq_len % 32 == 0 && rows >= 32 &&
                    aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
+  prm.z_stage = (a.z_map != nullptr && aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
   if (prm.tma_store) {
     ET_TRY(make_tmap_2d_sw64(&tz, a.Z, a.dtype, rows, (uint64_t)a.ld_z, (uint64_t)a.ld_z, 32, 32));
   } else {
