@@ -75,3 +75,16 @@ def test_col_linear_ffn_shape_gelu(etm):
     torch.cuda.synchronize()
     ref = oe.gelu(oe.linear(X, op.prune_col(Wnp, 0.8)["W_pruned"], b))
     assert_close(to64(Y), ref, what="col linear gelu")
+
+
+def test_col_linear_fully_pruned_is_bias(etm):
+    # degenerate case: every column pruned -> X_adjusted is all padding, Y = b exactly
+    dtype, M, d = "fp16", 256, 768
+    Wnp = make_matrix(48, (d, d), 0.05, dtype)
+    b = make_matrix(49, (d,), 0.02, dtype)
+    X = make_matrix(50, (M, d), 1.0, dtype)
+    cl = etm.ColLinear(dev_tensor(Wnp, dtype), 1.0)
+    assert cl.nk == 0 and cl.nk_pad == 64
+    Y = cl(dev_tensor(X, dtype), dev_tensor(b, dtype))
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(to64(Y), np.broadcast_to(b.astype(np.float64), (M, d)))
