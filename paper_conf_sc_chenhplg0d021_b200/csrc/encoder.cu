@@ -135,6 +135,11 @@ struct LnFuse {
 // the global mask restricted to the slice; the block computes heads h0..h1-1 only, the partial is
 // FP32 (reading C-21), and *bo_eff carries b_O only on the rank with h0 == 0 (plus this rank's
 // share of the pruned-V bias fold, reading C-6), so that the sum over ranks is the full output.
+// attention-aware Z without a memset: the 16-bit kernel's staged path (16-byte aligned Z rows)
+static bool zfill_ok(const et_attn_desc* d, const BlockWs& ws, int dq) {
+  return d->dtype != ET_FP32 && aligned16(ws.z) && (dq * 2) % 16 == 0;
+}
+
 et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et_packed_weight* wq,
                               const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
                               const void* bq, const void* bk, const void* bv, const void* bo, const BlockWs& ws,
@@ -152,8 +157,10 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
     ET_TRY(vprep_run(vp, st));
     bv_use = ws.bv_packed;
     *bo_eff = ws.bo_folded;
-    // pruned V features leave zero columns in Z (their constant b_V is folded into b_O')
-    ET_CUDA(cudaMemsetAsync(ws.z, 0, (size_t)M * dq * dtype_size(d->dtype), st));
+    // pruned V features leave zero columns in Z (their constant b_V is folded into b_O').  The 16-bit
+    // attention kernel's staged Z path writes whole head windows (zeros included, and empty heads
+    // zero theirs), so the memset is only needed for the FP32 kernel / unaligned Z.
+    if (!zfill_ok(d, ws, dq)) ET_CUDA(cudaMemsetAsync(ws.z, 0, (size_t)M * dq * dtype_size(d->dtype), st));
   }
   // 1. QKV projection: one launch, three segments; Q scaled by 1/sqrt(d_k) before rounding
   GemmArgs g{};
@@ -185,6 +192,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   a.Z = ws.z;
   a.ld_z = dq;
   a.z_map = rowv ? wv->row_map : nullptr;
+  a.z_fill_empty = rowv && zfill_ok(d, ws, dq) ? 1 : 0;
   a.lengths = d->lengths_dev;
   a.batch = d->batch;
   a.seq_len = d->seq_len;

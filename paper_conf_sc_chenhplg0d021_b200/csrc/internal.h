@@ -122,6 +122,7 @@ struct AttnArgs {
   float scale;
   et_dtype dtype;
   unsigned long long* ts;   // trace slot or nullptr
+  int z_fill_empty;         // z_map mode: heads with no kept V feature zero their Z window (replaces a Z memset)
 };
 et_status attention_run(const AttnArgs& a, cudaStream_t stream);
 et_status attention32_run(const AttnArgs& a, cudaStream_t stream);

@@ -72,6 +72,7 @@ struct AParams {
   int box_rows;             // TMA box height: min(128, total rows)
   int tma_store;            // Z written through TMA stores (dense V layout, seq_len % 32 == 0)
   int z_stage;              // z_map scatter staged in shared memory, stored as 16-byte row windows
+  int z_fill_empty;         // (with z_stage) a head with no kept V feature writes zeros over its Z window
   unsigned long long* ts;   // trace slot or nullptr
 };
 
@@ -116,7 +117,15 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
   const int hh = p.head_begin + blockIdx.y;
   const int vloc = p.v_col ? __ldg(p.v_col + hh) : hh * kDK;   // packed V column of this head
   const int vw = p.v_width ? __ldg(p.v_width + hh) : kDK;
-  if (vw == 0) {   // every V feature of the head pruned
+  if (vw == 0) {   // every V feature of the head pruned: Z = 0 there (reading C-6: b_V folded into b_O')
+    if (p.z_fill_empty) {   // the staged path writes every other head's whole window: no Z memset needed
+      using T0 = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
+      const int q0 = blockIdx.x * 128, nrow = min(128, p.S - q0);
+      constexpr int kU = kDK / 8;
+      for (int i = threadIdx.x; i < nrow * kU; i += blockDim.x)
+        *reinterpret_cast<uint4*>(static_cast<T0*>(p.Z) + (size_t)(blockIdx.z * p.S + q0 + i / kU) * p.ld_z +
+                                  (hh - p.head_begin) * kDK + (i % kU) * 8) = make_uint4(0, 0, 0, 0);
+    }
     trace_cta_end(p.ts);
     return;
   }
@@ -596,6 +605,7 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   prm.tma_store = (a.z_map == nullptr && a.v_width == nullptr && a.seq_len % 32 == 0 && rows >= 32 &&
                    aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
   prm.z_stage = (a.z_map != nullptr && aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
+  prm.z_fill_empty = prm.z_stage && a.z_fill_empty;
   if (prm.tma_store) {
     ET_TRY(make_tmap_2d_sw64(&tz, a.Z, a.dtype, rows, (uint64_t)a.ld_z, (uint64_t)a.ld_z, 32, 32));
   } else {

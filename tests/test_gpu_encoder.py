@@ -170,3 +170,17 @@ def test_fused_oproj_layernorm_path(etm, key, kw, monkeypatch):
     rdt = cfg.dtype
     Y, enc, _ = _gpu(etm, cfg, raws, X, lens, resid=rdt)
     assert_close(Y, _oracle(cfg, raws, X, lens), what=f"fused O-proj+LN {key} {kw}")
+
+
+def test_attention_aware_fully_pruned_head(etm):
+    # a head whose W_V rows are all pruned (reading C-6: Z = 0 there, b_V folded into b_O') in layer 1
+    # only: the Z buffer is reused across layers, so that head's window must be re-zeroed (the
+    # attention kernel writes it; there is no Z memset on the 16-bit path)
+    cfg, raws, X, lens = _case("C4", layers=2, batch=2)
+    raws[1]["wv"][64:128] *= 1e-3
+    info = oe.prune_layer(raws[1], cfg.scheme, cfg.ratio)[1]
+    assert info["wv"]["keep"][64:128].sum() == 0
+    assert oe.prune_layer(raws[0], cfg.scheme, cfg.ratio)[1]["wv"]["keep"][64:128].sum() > 0
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens)
+    ref = _oracle(cfg, raws, X, lens)
+    assert_close(Y.reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what="C4 with an empty V head")
