@@ -51,8 +51,10 @@ typedef enum { ET_FP16 = 0, ET_BF16 = 1, ET_FP32 = 2 } et_dtype;
 /* Pruning patterns (§4.1-4.2; attention-aware assignment line 107, 317). */
 typedef enum { ET_PRUNE_NONE = 0, ET_PRUNE_TILE = 1, ET_PRUNE_ROW = 2, ET_PRUNE_COL = 3 } et_pattern;
 
-/* Attention operator form (§3.2, switch at a length threshold line 244). */
-typedef enum { ET_ATTN_AUTO = 0, ET_ATTN_SHORT = 1, ET_ATTN_LONG = 2 } et_attn_mode;
+/* Attention operator form (§3.2, switch at a length threshold line 244).
+ * ET_ATTN_SHORT_GENERIC: the short form through its generic kernel even where the specialised
+ * S <= 128, d_k = 64 kernel applies (test hook: both kernels are checked against the oracle). */
+typedef enum { ET_ATTN_AUTO = 0, ET_ATTN_SHORT = 1, ET_ATTN_LONG = 2, ET_ATTN_SHORT_GENERIC = 3 } et_attn_mode;
 
 /* FFN activation ("an activation layer"; GELU(erf) for BERT, ReLU otherwise). */
 typedef enum { ET_ACT_GELU_ERF = 0, ET_ACT_RELU = 1 } et_act;
@@ -299,9 +301,8 @@ et_status et_trace_get(int32_t i, int32_t* kind, float* ms);
 /* Number of library kernels launched by this thread since process start (launch accounting). */
 int64_t et_launch_count(void);
 
-/* Diagnostics (not part of the metric): tcgen05 probe (profiles/r01/M1_tcgen05_probe.md). */
-int et_diag_mma_probe(const void* A, const void* B, float* D, int N, int a_mode, int b_mode, int iters, int n_acc,
-                      int issue_mode, long long* cycles, int grid, void* stream);
+/* Diagnostics (tcgen05 / TMA probes, profiles/r01/M1_tcgen05_probe.md, profiles/r02/) live in a
+ * separate libet_diag.so built from paper_conf_sc_chenhplg0d021_b200/diag/ (not part of this ABI). */
 
 #ifdef __cplusplus
 }

@@ -20,14 +20,14 @@ LIB_PATH = os.environ.get("ET_LIB_PATH") or os.path.join(_HERE, "libet.so")
 # enums (include/et.h)
 FP16, BF16, FP32 = 0, 1, 2
 PRUNE_NONE, PRUNE_TILE, PRUNE_ROW, PRUNE_COL = 0, 1, 2, 3
-ATTN_AUTO, ATTN_SHORT, ATTN_LONG = 0, 1, 2
+ATTN_AUTO, ATTN_SHORT, ATTN_LONG, ATTN_SHORT_GENERIC = 0, 1, 2, 3
 ACT_GELU_ERF, ACT_RELU = 0, 1
 EPI_BIAS, EPI_BIAS_SCALE, EPI_BIAS_GELU, EPI_BIAS_RELU, EPI_F32, EPI_PART16 = 0, 1, 2, 3, 4, 5
 
 _DT = {"fp16": FP16, "bf16": BF16, "fp32": FP32}
 _TORCH_DT = {FP16: torch.float16, BF16: torch.bfloat16, FP32: torch.float32}
 _PAT = {"none": PRUNE_NONE, "tile": PRUNE_TILE, "row": PRUNE_ROW, "col": PRUNE_COL}
-_MODE = {"auto": ATTN_AUTO, "short": ATTN_SHORT, "long": ATTN_LONG}
+_MODE = {"auto": ATTN_AUTO, "short": ATTN_SHORT, "long": ATTN_LONG, "short_generic": ATTN_SHORT_GENERIC}
 _ACT = {"gelu": ACT_GELU_ERF, "relu": ACT_RELU}
 
 
@@ -91,7 +91,7 @@ _short_max = _sig("et_attn_short_max", _i32, [_i32])
 
 SYMBOLS = ["et_last_error", "et_version", "et_prune_pack_query", "et_prune_pack", "et_unpack", "et_linear_fwd",
            "et_layernorm_fwd", "et_attn_short_max", "et_attn_core_fwd", "et_attention_workspace_size",
-           "et_attention_fwd", "et_encoder_workspace_size", "et_encoder_fwd", "et_diag_mma_probe"]
+           "et_attention_fwd", "et_encoder_workspace_size", "et_encoder_fwd"]
 
 
 def _check(st: int):
@@ -405,7 +405,7 @@ class Encoder:
     """A packed encoder stack bound to a fixed problem shape: owns the C layer array and workspace."""
 
     def __init__(self, layers: list, batch: int, seq_len: int, heads: int, d_ff: int, act="gelu", ln_eps=1e-12,
-                 dtype="fp16", resid_dtype="fp16", causal=False, mode="auto", lengths=None):
+                 dtype="fp16", resid_dtype=None, causal=False, mode="auto", lengths=None):
         self.layers = layers
         self.arr = (LayerC * len(layers))(*[l.c for l in layers])
         d_model = layers[0].packed["wq"].c.rows
@@ -413,7 +413,9 @@ class Encoder:
         self.desc = attn_desc(batch, seq_len, heads, d_model, dtype, lengths, causal, mode)
         self.lengths = lengths
         self.d_ff, self.act, self.eps = d_ff, _ACT[act], ln_eps
-        self.dtype, self.resid_dtype = dtype_code(dtype), dtype_code(resid_dtype)
+        # residual stream dtype (reading C-22): the operand dtype unless given (FP32 is the other choice)
+        self.dtype = dtype_code(dtype)
+        self.resid_dtype = self.dtype if resid_dtype is None else dtype_code(resid_dtype)
         nb = _sz()
         _check(_enc_ws(ctypes.byref(self.desc), len(layers), d_ff, self.resid_dtype, self.arr, ctypes.byref(nb)))
         self.ws = torch.empty(nb.value, dtype=torch.uint8, device="cuda")

@@ -20,9 +20,11 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
+DIAG = os.path.join(PKG, "diag")
 INCLUDE = os.path.join(ROOT, "include")
 BUILD = os.path.join(ROOT, "build", "et")
 LIB = os.path.join(PKG, "libet.so")
+DIAG_LIB = os.path.join(PKG, "libet_diag.so")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
@@ -44,6 +46,33 @@ def _headers() -> list[str]:
 
 def sources() -> list[str]:
     return sorted(glob.glob(os.path.join(CSRC, "**", "*.cu"), recursive=True))
+
+
+def diag_sources() -> list[str]:
+    return sorted(glob.glob(os.path.join(DIAG, "*.cu")))
+
+
+def build_diag(verbose: bool = False) -> str:
+    """Microbenchmark probes (diag/*.cu: M1 tcgen05 shapes, M1b issue / TMEM fill rates, TMA pull)
+    in their own libet_diag.so, linked against libet.so; never loaded by the product path."""
+    nvcc = _nvcc()
+    bdir = BUILD + "_diag"
+    os.makedirs(bdir, exist_ok=True)
+    hdr_mtime = max([os.path.getmtime(h) for h in _headers()] + [0.0])
+    objs = []
+    for src in diag_sources():
+        obj = os.path.join(bdir, os.path.basename(src) + ".o")
+        objs.append(obj)
+        if not os.path.exists(obj) or os.path.getmtime(obj) < max(os.path.getmtime(src), hdr_mtime):
+            r = subprocess.run([nvcc, *ARCH, *FLAGS, "-c", src, "-o", obj], capture_output=True, text=True)
+            if r.returncode != 0:
+                raise RuntimeError("compile failed: " + src + "\n" + r.stdout + r.stderr)
+    r = subprocess.run([nvcc, *ARCH, "-shared", "-o", DIAG_LIB, *objs, "-L", PKG, "-let", "-Xlinker",
+                        "-rpath=$ORIGIN", "-lcudart_static", "-ldl", "-lrt", "-lpthread"],
+                       capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError("link failed: " + r.stdout + r.stderr)
+    return DIAG_LIB
 
 
 def build(verbose: bool = False, force: bool = False, debug: bool = False, variant: str | None = None,
@@ -101,3 +130,5 @@ if __name__ == "__main__":
     var = sys.argv[sys.argv.index("--variant") + 1] if "--variant" in sys.argv else None
     defs = tuple(a[2:] for a in sys.argv if a.startswith("-D"))
     print(build(verbose=True, force="--force" in sys.argv, debug="--debug" in sys.argv, variant=var, defines=defs))
+    if "--diag" in sys.argv:
+        print(build_diag(verbose=True))

@@ -36,7 +36,7 @@ et_epilogue part_epi_of(et_dtype dt) { return dt == ET_FP16 ? ET_EPI_PART16 : ET
 bool long_form_for(const et_attn_desc* d) {
   const int dk = d->d_model / d->heads;
   if (d->mode == ET_ATTN_LONG) return true;
-  if (d->mode == ET_ATTN_SHORT) return false;
+  if (d->mode == ET_ATTN_SHORT || d->mode == ET_ATTN_SHORT_GENERIC) return false;
   return d->seq_len > attn_short_max(dk);
 }
 
@@ -50,19 +50,32 @@ et_status check_desc(const et_attn_desc* d) {
   const int dk = d->d_model / d->heads;
   if (dk != 64 && dk != 128) return fail(ET_ERR_UNSUPPORTED, "d_k must be 64 or 128 (got %d)", dk);
   if (d->d_model % 64) return fail(ET_ERR_UNSUPPORTED, "d_model must be a multiple of 64");
-  if (d->mode == ET_ATTN_SHORT && d->seq_len > attn_short_max(dk))
+  if (d->mode < ET_ATTN_AUTO || d->mode > ET_ATTN_SHORT_GENERIC) return fail(ET_ERR_INVALID_ARG, "bad attention mode %d", (int)d->mode);
+  if ((d->mode == ET_ATTN_SHORT || d->mode == ET_ATTN_SHORT_GENERIC) && d->seq_len > attn_short_max(dk))
     return fail(ET_ERR_UNSUPPORTED, "short attention form needs seq_len <= %d", attn_short_max(dk));
   if (d->head_begin < 0 || d->head_end > d->heads || d->head_begin >= d->head_end)
     return fail(ET_ERR_INVALID_ARG, "bad head range [%d, %d)", d->head_begin, d->head_end);
   return ET_OK;
 }
 
-et_status check_weight(const et_packed_weight* w, int rows, int cols, et_dtype dt, const char* name, bool allow_row) {
+et_status check_weight(const et_packed_weight* w, int rows, int cols, et_dtype dt, const char* name, bool allow_row,
+                       int dk = 0) {
   if (!w || !w->values) return fail(ET_ERR_INVALID_ARG, "%s: packed weight without values", name);
   if (w->rows != rows || w->cols != cols)
     return fail(ET_ERR_INVALID_ARG, "%s: shape %dx%d, expected %dx%d", name, w->rows, w->cols, rows, cols);
   if (w->dtype != dt) return fail(ET_ERR_INVALID_ARG, "%s: dtype mismatch", name);
   if (w->pattern == ET_PRUNE_ROW && !allow_row) return fail(ET_ERR_UNSUPPORTED, "%s: row pruning only for W_V", name);
+  if (w->pattern == ET_PRUNE_ROW) {
+    // the attention kernels read head h's V features from a window that starts on a 16-aligned packed
+    // column and map them back with row_map inside the head's own Z window: the packing must pad
+    // per head (group_rows = d_k, reading C-5), else columns of one head land in another's window
+    if (w->group_rows != dk)
+      return fail(ET_ERR_INVALID_ARG, "%s: row-pruned W_V must be packed with group_rows = d_k = %d (got %d)", name, dk,
+                  w->group_rows);
+    if (w->rows_padded % 16 || w->rows_padded < w->nnz || w->rows_padded > w->nnz + 15 * (rows / dk))
+      return fail(ET_ERR_INVALID_ARG, "%s: rows_padded %d inconsistent with %d kept rows in %d heads", name,
+                  w->rows_padded, w->nnz, rows / dk);
+  }
   if (w->pattern != ET_PRUNE_TILE && w->pattern != ET_PRUNE_ROW)
     return fail(ET_ERR_UNSUPPORTED, "%s: pattern %d not supported by the forward path", name, (int)w->pattern);
   return ET_OK;
@@ -135,11 +148,6 @@ struct LnFuse {
 // the global mask restricted to the slice; the block computes heads h0..h1-1 only, the partial is
 // FP32 (reading C-21), and *bo_eff carries b_O only on the rank with h0 == 0 (plus this rank's
 // share of the pruned-V bias fold, reading C-6), so that the sum over ranks is the full output.
-// attention-aware Z without a memset: the 16-bit kernel's staged path (16-byte aligned Z rows)
-static bool zfill_ok(const et_attn_desc* d, const BlockWs& ws, int dq) {
-  return d->dtype != ET_FP32 && aligned16(ws.z) && (dq * 2) % 16 == 0;
-}
-
 et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et_packed_weight* wq,
                               const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
                               const void* bq, const void* bk, const void* bv, const void* bo, const BlockWs& ws,
@@ -157,10 +165,8 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
     ET_TRY(vprep_run(vp, st));
     bv_use = ws.bv_packed;
     *bo_eff = ws.bo_folded;
-    // pruned V features leave zero columns in Z (their constant b_V is folded into b_O').  The 16-bit
-    // attention kernel's staged Z path writes whole head windows (zeros included, and empty heads
-    // zero theirs), so the memset is only needed for the FP32 kernel / unaligned Z.
-    if (!zfill_ok(d, ws, dq)) ET_CUDA(cudaMemsetAsync(ws.z, 0, (size_t)M * dq * dtype_size(d->dtype), st));
+    // pruned V features leave zero columns in Z (their constant b_V is folded into b_O'):
+    // attention_run guarantees them (a.z_clear below)
   }
   // 1. QKV projection: one launch, three segments; Q scaled by 1/sqrt(d_k) before rounding
   GemmArgs g{};
@@ -192,7 +198,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   a.Z = ws.z;
   a.ld_z = dq;
   a.z_map = rowv ? wv->row_map : nullptr;
-  a.z_fill_empty = rowv && zfill_ok(d, ws, dq) ? 1 : 0;
+  a.z_clear = rowv ? 1 : 0;
   a.lengths = d->lengths_dev;
   a.batch = d->batch;
   a.seq_len = d->seq_len;
@@ -202,6 +208,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   a.head_end = Hr;
   a.causal = d->causal;
   a.long_form = long_form_for(d) ? 1 : 0;
+  a.generic = d->mode == ET_ATTN_SHORT_GENERIC ? 1 : 0;
   a.v_width_max = dk;
   a.scale = 1.0f;
   a.dtype = d->dtype;
@@ -271,6 +278,7 @@ et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld
   a.head_end = desc->head_end;
   a.causal = desc->causal;
   a.long_form = long_form_for(desc) ? 1 : 0;
+  a.generic = desc->mode == ET_ATTN_SHORT_GENERIC ? 1 : 0;
   a.v_width_max = v_width ? v_width_max : dk;
   a.scale = scale;
   a.dtype = desc->dtype;
@@ -298,7 +306,7 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   if (hp && ln_gamma) return fail(ET_ERR_INVALID_ARG, "et_attention_fwd: head-parallel ranges take no LayerNorm (it follows the all-reduce)");
   ET_TRY(check_weight(wq, dq, dm, desc->dtype, "W_Q", false));
   ET_TRY(check_weight(wk, dq, dm, desc->dtype, "W_K", false));
-  ET_TRY(check_weight(wv, dq, dm, desc->dtype, "W_V", true));
+  ET_TRY(check_weight(wv, dq, dm, desc->dtype, "W_V", true, dm / desc->heads));
   ET_TRY(check_weight(wo, dm, dq, desc->dtype, "W_O", false));
   if (!X || !out || !workspace) return fail(ET_ERR_INVALID_ARG, "et_attention_fwd: null pointer");
   size_t need = 0;
@@ -367,7 +375,7 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     const et_layer& L = layers[l];
     ET_TRY(check_weight(&L.wq, dm, dm, desc->dtype, "W_Q", false));
     ET_TRY(check_weight(&L.wk, dm, dm, desc->dtype, "W_K", false));
-    ET_TRY(check_weight(&L.wv, dm, dm, desc->dtype, "W_V", true));
+    ET_TRY(check_weight(&L.wv, dm, dm, desc->dtype, "W_V", true, dm / desc->heads));
     ET_TRY(check_weight(&L.wo, dm, dm, desc->dtype, "W_O", false));
     ET_TRY(check_weight(&L.w1, d_ff, dm, desc->dtype, "W_1", false));
     ET_TRY(check_weight(&L.w2, dm, d_ff, desc->dtype, "W_2", false));

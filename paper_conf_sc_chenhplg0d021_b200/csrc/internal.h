@@ -122,7 +122,9 @@ struct AttnArgs {
   float scale;
   et_dtype dtype;
   unsigned long long* ts;   // trace slot or nullptr
-  int z_fill_empty;         // z_map mode: heads with no kept V feature zero their Z window (replaces a Z memset)
+  int z_clear;              // z_map mode: Z columns no kept V feature maps to must be zero afterwards
+                            // (attention_run zero-fills whole head windows or memsets Z; one place decides)
+  int generic;              // force the generic short-form kernel (ET_ATTN_SHORT_GENERIC test hook)
 };
 et_status attention_run(const AttnArgs& a, cudaStream_t stream);
 et_status attention32_run(const AttnArgs& a, cudaStream_t stream);
@@ -156,12 +158,6 @@ et_status gather_cols_run(const void* in, int rows, int ld_in, const int32_t* id
 // ---------------------------------------------------------------- tracing (api.cu)
 // Record a mark of `kind` on `stream` if tracing is enabled; counts one kernel launch.
 unsigned long long* trace_slot(int kind);
-
-// Diagnostic switches read from the environment (e.g. ET_ATTN_GENERIC=1: skip specialised kernels).
-inline bool getenv_flag(const char* name) {
-  const char* v = std::getenv(name);
-  return v != nullptr && v[0] != 0 && v[0] != '0';
-}
 
 // Launch with programmatic stream serialisation (PDL): the kernel may begin while the previous
 // kernel on the stream finishes; it must call pdl_wait() (ptx.cuh) before touching global data.

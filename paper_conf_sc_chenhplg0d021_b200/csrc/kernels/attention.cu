@@ -570,7 +570,17 @@ et_status launch(const CUtensorMap& tm, const CUtensorMap& tz, const AParams& pr
 
 int attn_short_max(int d_k) { return (d_k == 64 || d_k == 128) ? 256 : 0; }
 
+// z_map mode with z_clear: Z columns that no kept V feature maps to must read as zero afterwards.
+// Decided here, next to the kernel choice: the 16-bit generic kernel's staged Z path writes every
+// head's whole window (zeros included; heads with no kept feature zero theirs, z_fill_empty), any
+// other path gets a memset of Z first.
+static bool z_staged(const AttnArgs& a) {
+  return a.dtype != ET_FP32 && a.z_map != nullptr && aligned16(a.Z) && (a.ld_z * 2) % 16 == 0;
+}
+
 et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
+  if (a.z_map != nullptr && a.z_clear && !z_staged(a) && a.batch > 0 && a.seq_len > 0)
+    ET_CUDA(cudaMemsetAsync(a.Z, 0, (size_t)a.batch * a.seq_len * a.ld_z * dtype_size(a.dtype), stream));
   if (a.dtype == ET_FP32) return attention32_run(a, stream);   // FP32 validation build (CUDA cores)
   if (a.d_k != 64 && a.d_k != 128) return fail(ET_ERR_UNSUPPORTED, "attention: d_k must be 64 or 128 (got %d)", a.d_k);
   if (a.v_width_max <= 0 || a.v_width_max > a.d_k || a.v_width_max % 16)
@@ -578,7 +588,7 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   if (!a.long_form && a.seq_len > 256) return fail(ET_ERR_UNSUPPORTED, "attention: short form needs seq_len <= 256");
   if (a.batch <= 0 || a.seq_len <= 0 || a.head_end <= a.head_begin) return ET_OK;
   if (!aligned16(a.qkv) || (a.ld_qkv * 2) % 16) return fail(ET_ERR_INVALID_ARG, "attention: QKV not 16B aligned");
-  if (attention128_applies(a) && !getenv_flag("ET_ATTN_GENERIC")) return attention128_run(a, stream);
+  if (attention128_applies(a) && !a.generic) return attention128_run(a, stream);
   const uint64_t rows = (uint64_t)a.batch * a.seq_len;
   const uint32_t box_rows = rows < 128 ? (uint32_t)rows : 128u;
   CUtensorMap tm, tz;
@@ -604,8 +614,8 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
   // TMA stores of Z: dense per-head V, every 32-row group inside one sequence, Z 16-byte aligned
   prm.tma_store = (a.z_map == nullptr && a.v_width == nullptr && a.seq_len % 32 == 0 && rows >= 32 &&
                    aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
-  prm.z_stage = (a.z_map != nullptr && aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
-  prm.z_fill_empty = prm.z_stage && a.z_fill_empty;
+  prm.z_stage = z_staged(a) ? 1 : 0;
+  prm.z_fill_empty = prm.z_stage && a.z_clear;
   if (prm.tma_store) {
     ET_TRY(make_tmap_2d_sw64(&tz, a.Z, a.dtype, rows, (uint64_t)a.ld_z, (uint64_t)a.ld_z, 32, 32));
   } else {

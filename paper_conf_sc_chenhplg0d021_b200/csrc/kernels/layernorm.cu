@@ -278,9 +278,8 @@ __global__ void __launch_bounds__(512) layernorm_kernel(const LnArgs a) {
 
 template <int NCH, int DT, int RT, bool P16>
 et_status launch_np(const LnArgs& a, cudaStream_t stream) {
-  // rows per CTA (one warp each): ET_LN_THREADS (experiment knob; default 128 threads = 4 rows)
-  static const int env_threads = getenv("ET_LN_THREADS") ? atoi(getenv("ET_LN_THREADS")) : 128;
-  const int threads = (env_threads == 256 || env_threads == 512) ? env_threads : 128;
+  // rows per CTA (one warp each): 128 threads = 4 rows (256 / 512 measured no faster, round 1)
+  constexpr int threads = 128;
   const int blocks = (a.M * 32 + threads - 1) / threads;
   cudaError_t e = cudaSuccess;
   switch (a.nparts) {
@@ -320,10 +319,9 @@ et_status layernorm_run(const LnArgs& a, cudaStream_t stream) {
   if (a.N % 4 || a.N > 128 * 8)
     return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 4 and <= 1024 (got %d)", a.N);
   if (a.M <= 0) return ET_OK;
-  // 8-wide form (16-byte accesses) for up to ET_LN8_MAXNP partial inputs (more partials: the
-  // 4-wide form, whose smaller per-lane register footprint keeps more rows in flight)
-  static const int ln8_maxnp = getenv("ET_LN8_MAXNP") ? atoi(getenv("ET_LN8_MAXNP")) : 4;
-  if (a.N % 8 == 0 && a.nparts <= ln8_maxnp) {
+  // 8-wide form (16-byte accesses) for up to 4 partial inputs (more partials: the 4-wide form,
+  // whose smaller per-lane register footprint keeps more rows in flight)
+  if (a.N % 8 == 0 && a.nparts <= 4) {
     switch ((a.N + 255) / 256) {
       case 1: return launch_dt<-1>(a, stream);
       case 2: return launch_dt<-2>(a, stream);

@@ -831,7 +831,7 @@ et_status make_tmap_3d(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t col
 
 // kEpiLN plan: np equal pieces of R tile rows (R even, R <= kLnMaxRows, np <= kLnMaxCluster), the
 // np pieces of a token block forming one cluster; the largest np whose grid fits one wave.
-// OFF by default (ET_LN_FUSE=1 enables it): measured on C3 (profiles/r01/README.md, v4) the fused
+// OFF unless built with -DET_GEMM_LN_FUSE: measured on C3 (profiles/r01/README.md, v4) the fused
 // O-projection + LayerNorm takes 12.2 us against 6.0 + 5.5 us unfused — the 6-slot ring (the FP32
 // stash takes the rest of shared memory) delays the first MMA by ~1.5k cycles, the cluster's
 // slowest CTA gates the statistics exchange, and the tail (stats, DSMEM exchange, normalisation)
@@ -839,8 +839,11 @@ et_status make_tmap_3d(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t col
 static int ln_pieces(const GemmArgs& a) {
   if (a.epi != kEpiLN || (a.dtype != ET_FP16 && a.dtype != ET_BF16) || a.nseg != 1 || a.K > 768 ||
       !a.resid || !a.gamma || !a.beta || a.seg[0].out_col != 0 || a.ldy != a.seg[0].tile_rows * 16 ||
-      (a.ldy * 2) % 16 || !aligned16(a.resid) || !getenv_flag("ET_LN_FUSE"))
+      (a.ldy * 2) % 16 || !aligned16(a.resid))
     return 0;
+#ifndef ET_GEMM_LN_FUSE
+  return 0;   // experiment (compile-time switch, off): slower than GEMM + LayerNorm kernel, see below
+#endif
   const int rows = a.seg[0].tile_rows, mblocks = (a.M + 127) / 128;
   int best = 0;
   for (int np = 1; np <= kLnMaxCluster; ++np) {
@@ -993,7 +996,7 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   }
   dim3 grid(np, mblocks, kparts);
   const bool bf = a.dtype == ET_BF16;
-  switch (a.epi) {
+  switch ((int)a.epi) {
     case ET_EPI_BIAS: return bf ? launch_typed<ET_EPI_BIAS, true>(tm, tmy, prm, grid, stream)
                                 : launch_typed<ET_EPI_BIAS, false>(tm, tmy, prm, grid, stream);
     case ET_EPI_BIAS_SCALE: return bf ? launch_typed<ET_EPI_BIAS_SCALE, true>(tm, tmy, prm, grid, stream)
@@ -1006,7 +1009,7 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
                                : launch_typed<ET_EPI_F32, false>(tm, tmy, prm, grid, stream);
     case ET_EPI_PART16: return bf ? launch_typed<ET_EPI_PART16, true>(tm, tmy, prm, grid, stream)
                                   : launch_typed<ET_EPI_PART16, false>(tm, tmy, prm, grid, stream);
-    case (et_epilogue)kEpiLN: return bf ? launch_typed<kEpiLN, true>(tm, tmy, prm, grid, stream, (unsigned)ln_np)
+    case kEpiLN: return bf ? launch_typed<kEpiLN, true>(tm, tmy, prm, grid, stream, (unsigned)ln_np)
                                         : launch_typed<kEpiLN, false>(tm, tmy, prm, grid, stream, (unsigned)ln_np);
     default: break;
   }

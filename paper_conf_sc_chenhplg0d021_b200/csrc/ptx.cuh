@@ -79,6 +79,40 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 }
 #endif
 
+// try_wait without a suspend-time hint (the hardware's default time limit): for pipelines whose
+// stages hand over every few hundred cycles, where a parked waiter's wake-up latency would sit on
+// the critical path.
+__device__ __forceinline__ bool mbar_try_wait_nohint(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      " selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_fast(uint64_t* bar, uint32_t parity) {
+#ifdef ET_WATCHDOG
+  long long n = 0;
+  while (!mbar_try_wait_nohint(bar, parity)) {
+    if (++n == (1ll << 26)) {
+      printf("ET_WATCHDOG: mbarrier @smem %u parity %u block (%d,%d,%d) thread %d\n", smem_u32(bar), parity,
+             blockIdx.x, blockIdx.y, blockIdx.z, threadIdx.x);
+      asm volatile("trap;");
+    }
+  }
+#else
+  while (!mbar_try_wait_nohint(bar, parity)) {
+  }
+#endif
+}
+__device__ __forceinline__ void mbar_wait_fast_warp(uint64_t* bar, uint32_t parity) {
+  mbar_wait_fast(bar, parity);
+  __syncwarp();
+}
+
 // Warp-collective wait: every lane spins, then the warp reconverges.  Lanes can leave the spin loop
 // on different iterations; a diverged warp reaching an elect-wrapped tcgen05 issue takes ptxas'
 // BRA.DIV slow path and issues the instruction once per divergent group (duplicate MMAs).
@@ -164,6 +198,18 @@ __device__ __forceinline__ void bulk_load(void* smem_dst, const void* gsrc, uint
           smem_u32(smem_dst)),
       "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
+}
+
+// 256-bit global load / store (sm_100: LDG.256 / STG.256; 32-byte aligned): one whole sector
+__device__ __forceinline__ void ld_global_v8(const void* p, uint32_t (&w)[8]) {
+  asm volatile("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+               : "l"(p));
+}
+__device__ __forceinline__ void st_global_v8(void* p, const uint32_t* w) {
+  asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(w[0]), "r"(w[1]), "r"(w[2]),
+               "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
+               : "memory");
 }
 
 // ------------------------------------------------------------------ tcgen05: TMEM management

@@ -13,7 +13,7 @@
 // N=16 MMAs (one per 16x16 tile) reach the tcgen05 floor of 8 cycles.
 #include <cuda_runtime.h>
 #include <cstdint>
-#include "../ptx.cuh"
+#include "ptx.cuh"
 
 namespace et {
 

@@ -9,8 +9,8 @@
 #include <cuda_runtime.h>
 #include <cstdint>
 
-#include "../internal.h"
-#include "../ptx.cuh"
+#include "internal.h"
+#include "ptx.cuh"
 
 namespace et {
 et_status make_tmap_2d(CUtensorMap* tm, const void* base, et_dtype dtype, uint64_t rows, uint64_t cols,

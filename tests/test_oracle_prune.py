@@ -183,3 +183,39 @@ def test_mask_in_overrides_and_pruned_values_do_not_matter():
 def test_bad_shapes_rejected():
     with pytest.raises(ValueError):
         op.tile_scores(np.zeros((20, 16)), 16, 16)
+
+
+def _zero_structure(Wp, t=16):
+    """(all-zero rows, all-zero t x t blocks, blocks that are partly zero) of a pruned matrix."""
+    zr = int(np.sum(np.all(Wp == 0, axis=1)))
+    r, c = Wp.shape[0] // t, Wp.shape[1] // t
+    blocks = Wp.reshape(r, t, c, t).transpose(0, 2, 1, 3).reshape(r, c, t * t)
+    zb = int(np.sum(np.all(blocks == 0, axis=2)))
+    partial = int(np.sum(np.any(blocks == 0, axis=2) & ~np.all(blocks == 0, axis=2)))
+    return zr, zb, partial
+
+
+@pytest.mark.parametrize("scheme", ["attention-aware", "tile"])
+def test_pattern_assignment_per_matrix(scheme):
+    """The per-matrix pattern of oracle.prune_layer, read off the pruned weights themselves
+    (§5.3 (i): attention-aware = "row pruned for W_V on all encoder layers and
+    tensor tile pruned for other weights"; (iv): tile pruning for all weights).  Under
+    attention-aware pruning W_V (and only W_V) has exactly floor(p d + 0.5) all-zero ROWS whose
+    zeros cut across 16x16 tiles; W_Q, W_K, W_O, W_1, W_2 have exactly floor(p T + 0.5) all-zero
+    16x16 TILES and no other zeros.  Swapping any two table entries fails this test."""
+    from et_synth import CONFIGS, make_layer
+    from oracle.encoder import prune_layer
+    cfg = CONFIGS["C2"]            # d = 512, d_ff = 2048, p = 0.8
+    raw = make_layer(cfg, 0)
+    w, _ = prune_layer(raw, scheme, cfg.ratio)
+    d, f, p = cfg.d_model, cfg.d_ff, cfg.ratio
+    for name, (rows, cols) in {"wq": (d, d), "wk": (d, d), "wv": (d, d), "wo": (d, d), "w1": (f, d),
+                               "w2": (d, f)}.items():
+        zr, zb, partial = _zero_structure(w[name])
+        if scheme == "attention-aware" and name == "wv":
+            assert zr == math.floor(p * rows + 0.5), name          # row pattern: whole rows gone
+            assert partial > 0, name                                # ... that do not align with tiles
+        else:
+            T = (rows // 16) * (cols // 16)
+            assert zb == math.floor(p * T + 0.5), name               # tile pattern: whole tiles gone
+            assert partial == 0 and zr == 0, name                   # ... and nothing else

@@ -12,7 +12,7 @@ import numpy as np
 import torch
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-lib = ctypes.CDLL(os.path.join(ROOT, "paper_conf_sc_chenhplg0d021_b200", "libet.so"))
+lib = ctypes.CDLL(os.path.join(ROOT, "paper_conf_sc_chenhplg0d021_b200", "libet_diag.so"))
 lib.et_diag_mma_probe.argtypes = [ctypes.c_void_p] * 3 + [ctypes.c_int] * 6 + [ctypes.c_void_p, ctypes.c_int,
                                                                             ctypes.c_void_p]
 

@@ -4,7 +4,8 @@ import ctypes, sys
 import numpy as np, torch
 sys.path.insert(0, '.')
 import paper_conf_sc_chenhplg0d021_b200 as et
-f = et._lib.et_diag_tma_probe
+import os
+f = ctypes.CDLL(os.path.join(os.path.dirname(et.__file__), "libet_diag.so")).et_diag_tma_probe
 f.restype = ctypes.c_int
 f.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p]
 for grid in (128, 148):
