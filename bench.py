@@ -54,6 +54,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-parity", action="store_true", help="skip the sampled oracle comparison in the line")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the cpu_baseline sample")
+    ap.add_argument("--scaling", choices=["weak", "strong"], default=None,
+                    help="weak: every rank runs the config's batch (default; C3 metric); strong: the config's "
+                         "batch is the global batch, split over the ranks (default for C5: B = 256 / N)")
     ap.add_argument("--parallel", choices=["batch", "head"], default="batch",
                     help="batch: batch sharding (default, weak scaling); head: head-parallel latency mode "
                          "(Eq. 4 partials + NCCL all-reduce per layer, strong scaling)")
@@ -188,35 +191,33 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------------------ roofline model
-def kernel_model(cfg, nnz: dict, kparts2: int, es: int, resid_es: int, ps: int):
-    """Algorithmic bytes and (effective) FLOPs of ONE launch of each kernel kind for one layer of
-    `cfg`.  nnz: kept 16x16 tiles per matrix; ps: bytes per partial-sum
-    element handed to the LayerNorm kernels (2 on the FP16 path, 4 on BF16)."""
+STEP_OF_KERNEL = {"qkv_gemm": "qkv", "attention": "attention", "oproj_gemm": "oproj_ln", "ln1": "oproj_ln",
+                  "ffn1_gemm": "ffn1", "ffn2_gemm": "ffn2_ln", "ln2": "ffn2_ln"}
+
+
+def step_model(cfg, nnz: dict, v_kept: int | None, es: int):
+    """algorithmic bytes and effective FLOPs of one layer's five steps
+    (whole batch).  Bytes = read the step's inputs + its kept weights + write its outputs once, in the
+    storage dtype (es bytes; the residual stream counted like the activations, as in Appendix B);
+    FLOPs = 2 M x kept weights (16x16 tiles, or kept W_V rows) + attention on unmasked (q, k) pairs,
+    P.V over the kept V features.  nnz: kept tiles per tile-pruned matrix; v_kept: kept W_V rows when
+    W_V is row-pruned (else None)."""
     M, d, f, H, S, B = cfg.tokens, cfg.d_model, cfg.d_ff, cfg.heads, cfg.seq_len, cfg.batch
     dk = d // H
-    t = 512   # bytes per packed 16x16 fp16/bf16 tile
-    mm = lambda n: 2.0 * M * 256 * n          # one MMA tile = 16x16 weights against M tokens
-    pairs = B * H * (S * (S + 1) / 2 if cfg.causal else S * S)
+    t = 256 * es                                      # bytes of one kept 16x16 tile
+    mm = lambda n: 2.0 * M * 256 * n                 # noqa: E731  one tile against M tokens
+    pairs = B * (S * (S + 1) / 2 if cfg.causal else S * S)   # unmasked (q, k) pairs per head (lengths = S)
+    vw = v_kept if v_kept is not None else d          # V width the attention moves / multiplies
+    wv_b = v_kept * d * es if v_kept is not None else nnz["wv"] * t
+    wv_f = 2.0 * M * v_kept * d if v_kept is not None else mm(nnz["wv"])
     return {
-        "qkv_gemm": (M * d * es + (nnz["wq"] + nnz["wk"] + nnz["wv"]) * t + M * 3 * d * es,
-                     mm(nnz["wq"] + nnz["wk"] + nnz["wv"])),
-        "attention": (M * 3 * d * es + M * d * es, 4.0 * pairs * dk),
-        "oproj_gemm": (M * d * es + nnz["wo"] * t + M * d * ps, mm(nnz["wo"])),
-        "ln1": (M * d * ps + M * d * resid_es + M * d * es, 0.0),
-        "ffn1_gemm": (M * d * es + nnz["w1"] * t + M * f * es, mm(nnz["w1"])),
-        "ffn2_gemm": (M * f * es + nnz["w2"] * t + kparts2 * M * d * ps, mm(nnz["w2"])),
-        "ln2": (kparts2 * M * d * ps + M * d * resid_es + M * d * resid_es, 0.0),
+        "qkv": (M * d * es + (nnz["wq"] + nnz["wk"]) * t + wv_b + M * (2 * d + vw) * es,
+                mm(nnz["wq"] + nnz["wk"]) + wv_f),
+        "attention": (M * (2 * d + vw) * es + M * d * es, 2.0 * pairs * H * dk + 2.0 * pairs * vw),
+        "oproj_ln": (M * d * es + nnz["wo"] * t + M * d * es + M * d * es, mm(nnz["wo"])),
+        "ffn1": (M * d * es + nnz["w1"] * t + M * f * es, mm(nnz["w1"])),
+        "ffn2_ln": (M * f * es + nnz["w2"] * t + M * d * es + M * d * es, mm(nnz["w2"])),
     }
-
-
-def eff_flops_per_step(cfg, nnz_layers):
-    """North-star numerator: FLOPs on kept tiles + attention on unmasked pairs, all layers."""
-    tot = 0.0
-    M, H, S, B, d = cfg.tokens, cfg.heads, cfg.seq_len, cfg.batch, cfg.d_model
-    pairs = B * H * (S * (S + 1) / 2 if cfg.causal else S * S)
-    for nz in nnz_layers:
-        tot += 2.0 * M * 256 * sum(nz.values()) + 4.0 * pairs * (d // H)
-    return tot
 
 
 # ------------------------------------------------------------------------------------------ CPU oracle
@@ -290,7 +291,7 @@ def reference_arm(args):
     lens = make_lengths(cfg, ragged=False)
     from oracle import encoder as oe
     layers = [oe.prune_layer(r, cfg.scheme, cfg.ratio)[0] for r in raws]
-    per_step = 2
+    per_step = 1 if cfg.seq_len > 512 else 2
     for w in range(args.warmup):
         idx = np.arange(w * per_step, (w + 1) * per_step) % cfg.batch
         oe.encoder(X[idx].astype(np.float64), layers, cfg.heads, lens[idx], cfg.causal, cfg.act, cfg.ln_eps)
@@ -335,9 +336,15 @@ def our_arm(args):
 
     from paper_conf_sc_chenhplg0d021_b200.dist import shard_range
     base = CONFIGS[args.config]
-    cfg = base                                   # per-rank shard: the config's batch (weak scaling)
-    gcfg = base.with_(batch=base.batch * world)  # the global batch, generated identically everywhere
-    dtype = cfg.dtype if cfg.dtype != "fp32" else "fp16"
+    strong = (args.scaling == "strong") if args.scaling else base.name == "C5"
+    if strong:   # the config's batch is the global batch (C5: 256 sequences over N GPUs)
+        if base.batch % world:
+            raise SystemExit(f"bench.py: global batch {base.batch} does not split over {world} ranks")
+        cfg, gcfg = base.with_(batch=base.batch // world), base
+    else:        # every rank runs the config's batch
+        cfg, gcfg = base, base.with_(batch=base.batch * world)
+    dtype = cfg.dtype                            # C1: fp32 (the validation build, its BASELINE precision)
+    rdt = dtype if cfg.resid == "same" else cfg.resid   # residual-stream dtype (reading C-22)
     raws = [make_layer(cfg, l) for l in range(cfg.layers)]
     Xg = make_x(gcfg)
     b0, b1 = shard_range(gcfg.batch, world, rank)
@@ -345,11 +352,17 @@ def our_arm(args):
     lens = make_lengths(cfg, ragged=False)
 
     layers = [et.pack_layer(r, cfg.scheme, cfg.ratio, cfg.heads, dtype) for r in raws]
-    nnz_layers = [{n: l.packed[n].c.ntiles for n in ("wq", "wk", "wv", "wo", "w1", "w2")} for l in layers]
+    if world > 1:   # every rank packed the same masks (deterministic pack): checked, not assumed
+        from paper_conf_sc_chenhplg0d021_b200.dist import all_equal_across_ranks, layers_digest
+        if not all_equal_across_ranks(layers_digest(layers)):
+            raise SystemExit("bench.py: ranks packed different masks")
+    # kept 16x16 tiles per tile-pruned matrix; kept W_V rows (not padded tiles) when row-pruned
+    nnz_layers = [{n: l.packed[n].c.nnz for n in ("wq", "wk", "wv", "wo", "w1", "w2")} for l in layers]
+    vkept_layers = [l.packed["wv"].c.nnz if cfg.scheme == "attention-aware" else None for l in layers]
     L = torch.from_numpy(lens).cuda()
     enc = et.Encoder(layers, cfg.batch, cfg.seq_len, cfg.heads, cfg.d_ff, act=cfg.act, ln_eps=cfg.ln_eps,
-                     dtype=dtype, resid_dtype=dtype, causal=cfg.causal, mode=cfg.attn_mode, lengths=L)
-    tdt = et.torch_dtype(dtype)
+                     dtype=dtype, resid_dtype=rdt, causal=cfg.causal, mode=cfg.attn_mode, lengths=L)
+    tdt = et.torch_dtype(rdt)
     Xd = torch.from_numpy(np.ascontiguousarray(X.reshape(cfg.tokens, cfg.d_model))).cuda().to(tdt)
     out = torch.empty_like(Xd)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
@@ -493,52 +506,64 @@ def our_arm(args):
         pk = peaks()
         total_seqs = cfg.batch * world * K
         value = total_seqs / t_max
-        es = 2
-        model = kernel_model(cfg, nnz_layers[0], layers[0].packed["w2"].c.kparts, es, es, 2 if dtype == "fp16" else 4)
-        # dominant kernel: largest share of the traced step time
+        es = 4 if dtype == "fp32" else 2
+        models = [step_model(cfg, nz, vk, es) for nz, vk in zip(nnz_layers, vkept_layers)]
+        # dominant kernel: largest share of the traced step time; its SURVEY §8(d) step's algorithmic
+        # bytes / FLOPs over the step's kernels' average device spans (the O-projection and FFN2 steps
+        # include their LayerNorm kernel: "O proj + res + LN", "FFN2 + res + LN")
         tot = {k: sum(v) for k, v in per_kind.items()}
         dom = max(tot, key=tot.get) if tot else None
         roof = None
-        if dom and dom in model:
-            avg_s = statistics.mean(per_kind[dom]) / 1e3
-            nbytes, nflops = model[dom]
+        if dom and dom in STEP_OF_KERNEL:
+            step = STEP_OF_KERNEL[dom]
+            kerns = [k for k, st in STEP_OF_KERNEL.items() if st == step and k in per_kind]
+            avg_s = sum(statistics.mean(per_kind[k]) for k in kerns) / 1e3
+            nbytes, nflops = models[0][step]
             t_hbm = nbytes / (pk["hbm_gbs"] * 1e9)
-            t_tc = nflops / (pk["bf16_tflops_sustained"] * 1e12)
+            t_tc = nflops / (pk["bf16_tflops"] * 1e12)
             traffic = None
             tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
             if os.path.exists(tf):
                 with open(tf) as fh:
-                    traffic = json.load(fh).get(dom)
+                    tj = json.load(fh)
+                if all(k in tj for k in kerns):
+                    traffic = sum(tj[k] for k in kerns)
+            name = "+".join(kerns)
+            if dtype == "fp32":   # the validation build runs on the CUDA cores: report the HBM line
+                t_tc = 0.0
             if t_tc > t_hbm:
                 ach = nflops / avg_s / 1e12
-                roof = {"bound": "tensor", "achieved": ach, "peak": pk["bf16_tflops_sustained"], "unit": "TFLOP/s",
-                        "frac": ach / pk["bf16_tflops_sustained"], "traffic": traffic, "kernel": dom,
+                roof = {"bound": "tensor", "achieved": ach, "peak": pk["bf16_tflops"], "unit": "TFLOP/s",
+                        "frac": ach / pk["bf16_tflops"], "traffic": traffic, "kernel": name, "step": step,
                         "algorithmic_flops_per_launch": nflops, "avg_launch_ms": avg_s * 1e3,
-                        "peak_src": pk["src"] + " bf16_tflops_sustained (fp16 dense = bf16 dense)"}
+                        "peak_src": pk["src"] + " bf16_tflops (burst; fp16 dense = bf16 dense)"}
             else:
                 ach = nbytes / avg_s / 1e9
                 roof = {"bound": "hbm", "achieved": ach, "peak": pk["hbm_gbs"], "unit": "GB/s",
-                        "frac": ach / pk["hbm_gbs"], "traffic": traffic, "kernel": dom,
+                        "frac": ach / pk["hbm_gbs"], "traffic": traffic, "kernel": name, "step": step,
                         "algorithmic_bytes_per_launch": nbytes, "avg_launch_ms": avg_s * 1e3,
                         "peak_src": pk["src"] + " hbm_gbs"}
         share = {k: round(v / sum(tot.values()), 4) for k, v in tot.items()} if tot else {}
         kern_ms = {k: round(statistics.mean(v), 5) for k, v in per_kind.items()}
-        # stepwise roofline: sum over the layer's kernels of max(F/P_tc, B/P_hbm)
-        t_roof = cfg.layers * sum(max(f / (pk["bf16_tflops_sustained"] * 1e12), b / (pk["hbm_gbs"] * 1e9))
-                                  for b, f in model.values() if (b, f) != (0, 0))
-        eflops = eff_flops_per_step(cfg, nnz_layers) * world
-        ns = {"eff_tflops": eflops * K / t_max / 1e12}
-        ns["frac_of_measured_tc"] = ns["eff_tflops"] / pk["bf16_tflops"]
+        # stepwise roofline: sum over layers and steps of max(F / P_tc, B / P_hbm),
+        # on the algorithmic bytes of Appendix B, divided by the measured step time
+        t_roof = sum(max(f / (pk["bf16_tflops"] * 1e12), b / (pk["hbm_gbs"] * 1e9))
+                     for m in models for b, f in m.values())
+        eflops = sum(f for m in models for _, f in m.values()) * world
+        ns = {"eff_gflop_per_step": eflops / 1e9, "eff_tflops": eflops * K / t_max / 1e12}
+        ns["frac_of_measured_tc_burst"] = ns["eff_tflops"] / pk["bf16_tflops"]
+        ns["frac_of_measured_tc_sustained"] = ns["eff_tflops"] / pk["bf16_tflops_sustained"]
         ns["frac_of_spec_tc"] = ns["eff_tflops"] / SPEC_TC_TFLOPS
+        ns["target_frac"] = 0.60
         line = {
             "metric": METRIC, "value": value, "unit": "seqs/s", "n_gpus": world, "steps": K,
             "warmup": max(args.warmup, 3), "ms_per_step": 1e3 * t_max / K, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": dtype, "data": "synthetic",
-            "config": {"workload": workload_name(cfg), "global_batch": cfg.batch * world,
+            "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": dtype, "data": "synthetic",
+            "config": {"workload": workload_name(gcfg if strong else cfg), "global_batch": cfg.batch * world,
                        "seq_len": cfg.seq_len, "per_gpu_batch": cfg.batch,
                        "parallelism": f"dp{world} (batch sharded, no data-path collective)",
                        "l2": "flushed before every timed step (256 MiB write, outside the events)",
-                       "residual_stream": dtype, "attention_form": "short" if cfg.seq_len <= 256 else "long"},
+                       "residual_stream": rdt, "attention_form": "short" if cfg.seq_len <= 256 else "long"},
             "roofline": roof,
             "kernel_ms": kern_ms, "kernel_share": share,
             "north_star": ns,
@@ -547,6 +572,8 @@ def our_arm(args):
             "step_ms_p50": statistics.median(step_ms),
             "step_ms_p10": float(np.percentile(step_ms, 10)), "step_ms_p90": float(np.percentile(step_ms, 90)),
             "stepwise_roofline_frac": t_roof / (t_max / K),
+            "stepwise_roofline_ms": t_roof * 1e3,
+            "stepwise_bytes_per_layer": sum(b for b, _ in models[0].values()),
             "git": git_sha(),
             "traced_step_ms_p50": statistics.median(tr_ms),
             "launch": "one CUDA graph replay per step (et_encoder_graph_create / et_graph_launch)",
@@ -560,7 +587,7 @@ def our_arm(args):
         if not args.no_parity:
             line["parity"] = parity_sample(cfg, raws, X, lens, out, layers)
         if world == 1 and not args.no_cpu_baseline:
-            v, n, el = oracle_seqs_per_s(cfg, raws, X, lens, args.cpu_seconds, chunk=2)
+            v, n, el = oracle_seqs_per_s(cfg, raws, X, lens, args.cpu_seconds, chunk=1 if cfg.seq_len > 512 else 2)
             line["cpu_baseline"] = {"value": v, "unit": "seqs/s", "cores": cpu_threads(), "kind": "oracle",
                                     "sample": f"{n} sequences of {args.config} (all {cfg.layers} layers, float64 "
                                               f"numpy oracle, {el:.1f} s)"}

@@ -45,6 +45,16 @@ def mask_digest(words) -> str:
     return hashlib.sha256(memoryview(words).tobytes()).hexdigest()
 
 
+def layers_digest(layers) -> str:
+    """Digest over every packed mask of every layer (et.Layer objects): batch-sharded ranks pack the same
+    weights deterministically, and bench.py checks that the digests agree before timing."""
+    h = hashlib.sha256()
+    for lay in layers:
+        for n in ("wq", "wk", "wv", "wo", "w1", "w2"):
+            h.update(mask_digest(lay.packed[n].mask()).encode())
+    return h.hexdigest()
+
+
 def all_equal_across_ranks(digest: str) -> bool:
     """True iff every rank passed the same digest."""
     import torch.distributed as dist

@@ -27,8 +27,9 @@ def _oracle(cfg, raws, X, lens, idx=None):
     return oe.encoder(Xs.astype(np.float64), layers, cfg.heads, ls, cfg.causal, cfg.act, cfg.ln_eps)
 
 
-def _gpu(etm, cfg, raws, X, lens, resid="same", mode="auto"):
+def _gpu(etm, cfg, raws, X, lens, resid=None, mode="auto"):
     dtype = cfg.dtype
+    resid = cfg.resid if resid is None else resid
     rdt = dtype if resid == "same" else resid
     layers = [etm.pack_layer(r, cfg.scheme, cfg.ratio, cfg.heads, dtype) for r in raws]
     L = torch.from_numpy(lens).cuda()
@@ -91,9 +92,21 @@ def _full_depth(etm, key, batch, idx):
 
 
 def test_c5_full_depth_sampled(etm):
-    """C5 at full depth: 12 layers, S = 2048, long-form attention, FP16 residual stream; sampled
-    sequences 0 (len S) and 1 (len 1).  The tightest parity case of the configs (reading C-22)."""
-    _full_depth(etm, "C5", 4, np.array([0, 1]))
+    """C5 at full depth: 12 layers, S = 2048, long-form attention, in its run configuration (FP32
+    residual stream, reading C-22); sampled sequences 0 (len S) and 1 (len 1).  Held to 5e-3 max-abs,
+    4x inside the bar (measured 7.1e-4)."""
+    err, rel = _full_depth(etm, "C5", 4, np.array([0, 1]))
+    assert err <= 5e-3, err
+
+
+def test_c5_full_depth_fp16_residual_within_bar(etm):
+    """The same with an FP16 residual stream: inside the north-star bar (measured max-abs 0.019 of
+    0.02) — the reason C5 runs with the FP32 stream."""
+    cfg, raws, X, lens = _case("C5", batch=4)
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens, resid="same")
+    idx = np.array([0, 1])
+    ref = _oracle(cfg, raws, X, lens, idx)
+    assert_close(Y[idx].reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what="C5 fp16 residual")
 
 
 def test_c4_full_depth_sampled(etm):
