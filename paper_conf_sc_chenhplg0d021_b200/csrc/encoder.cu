@@ -94,6 +94,24 @@ GemmSegment seg_of(const et_packed_weight* w, const void* bias, int out_col) {
   return s;
 }
 
+// Tile rows [r0, r0 + n) of a packed weight as a GEMM segment (a head range of W_Q / W_K / W_V):
+// row_ptr advanced to row r0 with the weight's own K-part stride, bias advanced to feature 16 r0.
+GemmSegment seg_slice(const et_packed_weight* w, const void* bias, int out_col, int r0, int n) {
+  GemmSegment s = seg_of(w, bias, out_col);
+  s.rp_stride = s.tile_rows + 1;
+  s.row_ptr = w->part_row_ptr + r0;
+  s.tile_rows = n;
+  if (bias) s.bias = static_cast<const uint8_t*>(bias) + (size_t)r0 * 16 * dtype_size(w->dtype);
+  return s;
+}
+
+// Head-parallel call on the FULL packed weights (et.h: the library slices them): W_Q / W_K /
+// W_V rows of the range are tile-row slices; a row-pruned W_V is projected whole (its per-head
+// packed offsets live on the device); W_O runs over a full-width Z that is zero outside the range.
+bool full_weights(const et_attn_desc* d, const et_packed_weight* wq) {
+  return (d->head_begin != 0 || d->head_end != d->heads) && wq && wq->rows == d->d_model;
+}
+
 // Workspace of one attention block (shared by the encoder).
 struct BlockWs {
   void* qkv;        // [M, ldq]
@@ -115,13 +133,13 @@ int v_cols_of(const et_packed_weight* wv, int d) {   // d: the width W_V produce
 int inner_width(const et_attn_desc* d) { return (d->head_end - d->head_begin) * (d->d_model / d->heads); }
 bool head_parallel(const et_attn_desc* d) { return d->head_begin != 0 || d->head_end != d->heads; }
 
-void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, BlockWs* ws) {
+void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, BlockWs* ws, bool zfull = false) {
   const size_t M = (size_t)d->batch * d->seq_len;
   const size_t es = dtype_size(d->dtype);
   const int dq = inner_width(d);
   ws->ldq = 2 * dq + vmax;
   ws->qkv = c.take(M * ws->ldq * es);
-  ws->z = c.take(M * dq * es);
+  ws->z = c.take(M * (zfull ? d->d_model : dq) * es);
   ws->part = c.take((size_t)kparts_max * M * d->d_model * 4);   // sized for FP32
   ws->v_col = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
   ws->v_width = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
@@ -157,11 +175,16 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   const int Hr = d->head_end - d->head_begin, dq = Hr * dk;
   const int M = d->batch * d->seq_len;
   const bool rowv = wv->pattern == ET_PRUNE_ROW;
+  const bool full = full_weights(d, wq);
+  const int h0 = d->head_begin;
+  const int r0 = full ? h0 * dk / 16 : 0, nr = dq / 16;   // the range's tile rows of W_Q / W_K / W_V
   const void* bo_rank = (hp && d->head_begin != 0) ? nullptr : bo;   // b_O enters the sum once
   const void* bv_use = bv;
   *bo_eff = bo_rank;
   if (rowv) {
-    VPrep vp{wv, wo, bv, bo_rank, Hr, dk, d->dtype, ws.v_col, ws.v_width, ws.bv_packed, ws.bo_folded};
+    // full weights: every head's packed V columns, and the fold over this range's features only
+    VPrep vp{wv, wo, bv, bo_rank, full ? d->heads : Hr, dk, full ? h0 * dk : 0, full ? h0 * dk + dq : dq,
+             d->dtype, ws.v_col, ws.v_width, ws.bv_packed, ws.bo_folded};
     ET_TRY(vprep_run(vp, st));
     bv_use = ws.bv_packed;
     *bo_eff = ws.bo_folded;
@@ -176,11 +199,11 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   g.ldx = dm;
   g.dtype = d->dtype;
   g.nseg = 3;
-  g.seg[0] = seg_of(wq, bq, 0);
+  g.seg[0] = full ? seg_slice(wq, bq, 0, r0, nr) : seg_of(wq, bq, 0);
   g.seg[0].apply_scale = 1;
   g.seg[0].scale = 1.0f / std::sqrt((float)dk);
-  g.seg[1] = seg_of(wk, bk, dq);
-  g.seg[2] = seg_of(wv, bv_use, 2 * dq);
+  g.seg[1] = full ? seg_slice(wk, bk, dq, r0, nr) : seg_of(wk, bk, dq);
+  g.seg[2] = (full && !rowv) ? seg_slice(wv, bv_use, 2 * dq, r0, nr) : seg_of(wv, bv_use, 2 * dq);
   g.Y = ws.qkv;
   g.ldy = ws.ldq;
   g.epi = ET_EPI_BIAS_SCALE;
@@ -193,11 +216,16 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   a.q_off = 0;
   a.k_off = dq;
   a.v_off = 2 * dq;
-  a.v_col = rowv ? ws.v_col : nullptr;
-  a.v_width = rowv ? ws.v_width : nullptr;
+  a.v_col = rowv ? ws.v_col + (full ? h0 : 0) : nullptr;
+  a.v_width = rowv ? ws.v_width + (full ? h0 : 0) : nullptr;
   a.Z = ws.z;
   a.ld_z = dq;
   a.z_map = rowv ? wv->row_map : nullptr;
+  if (full) {   // Z full width, zero outside this range's heads (W_O runs over all its columns)
+    ET_CUDA(cudaMemsetAsync(ws.z, 0, (size_t)M * dm * dtype_size(d->dtype), st));
+    a.ld_z = dm;
+    if (!rowv) a.Z = static_cast<uint8_t*>(ws.z) + (size_t)h0 * dk * dtype_size(d->dtype);   // row_map is global
+  }
   a.z_clear = rowv ? 1 : 0;
   a.lengths = d->lengths_dev;
   a.batch = d->batch;
@@ -218,8 +246,8 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   GemmArgs o{};
   o.X = ws.z;
   o.M = M;
-  o.K = dq;
-  o.ldx = dq;
+  o.K = full ? dm : dq;
+  o.ldx = full ? dm : dq;
   o.dtype = d->dtype;
   o.nseg = 1;
   o.seg[0] = seg_of(wo, nullptr, 0);
@@ -290,7 +318,8 @@ et_status et_attention_workspace_size(const et_attn_desc* desc, const et_packed_
   if (!wv || !bytes) return fail(ET_ERR_INVALID_ARG, "et_attention_workspace_size: null pointer");
   Carver c{nullptr};
   BlockWs ws;
-  carve_block(c, desc, v_cols_of(wv, inner_width(desc)), 1, &ws);
+  const bool full = head_parallel(desc) && wv->rows == desc->d_model;
+  carve_block(c, desc, v_cols_of(wv, full ? desc->d_model : inner_width(desc)), 1, &ws, full);
   *bytes = c.off + 256;
   return ET_OK;
 }
@@ -304,10 +333,15 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   const int dm = desc->d_model, dq = inner_width(desc);
   const bool hp = head_parallel(desc);
   if (hp && ln_gamma) return fail(ET_ERR_INVALID_ARG, "et_attention_fwd: head-parallel ranges take no LayerNorm (it follows the all-reduce)");
-  ET_TRY(check_weight(wq, dq, dm, desc->dtype, "W_Q", false));
-  ET_TRY(check_weight(wk, dq, dm, desc->dtype, "W_K", false));
-  ET_TRY(check_weight(wv, dq, dm, desc->dtype, "W_V", true, dm / desc->heads));
-  ET_TRY(check_weight(wo, dm, dq, desc->dtype, "W_O", false));
+  // head range on the full weights (the library slices them), or on the caller's slices
+  const bool full = full_weights(desc, wq);
+  const int wr = full ? dm : dq;
+  ET_TRY(check_weight(wq, wr, dm, desc->dtype, "W_Q", false));
+  ET_TRY(check_weight(wk, wr, dm, desc->dtype, "W_K", false));
+  ET_TRY(check_weight(wv, wr, dm, desc->dtype, "W_V", true, dm / desc->heads));
+  ET_TRY(check_weight(wo, dm, wr, desc->dtype, "W_O", false));
+  if (full && (dq % 16 || (desc->head_begin * (dm / desc->heads)) % 16))
+    return fail(ET_ERR_UNSUPPORTED, "et_attention_fwd: head range must start on a 16-row tile boundary");
   if (!X || !out || !workspace) return fail(ET_ERR_INVALID_ARG, "et_attention_fwd: null pointer");
   size_t need = 0;
   ET_TRY(et_attention_workspace_size(desc, wv, &need));
@@ -315,7 +349,7 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   Carver c{static_cast<uint8_t*>(workspace)};
   BlockWs ws;
-  carve_block(c, desc, v_cols_of(wv, dq), 1, &ws);
+  carve_block(c, desc, v_cols_of(wv, full ? dm : dq), 1, &ws, full);
   const void* bo_eff = bo;
   LnFuse lf{X, ln_gamma, ln_beta, ln_eps, out, false};
   ET_TRY(run_attention_block(desc, X, wq, wk, wv, wo, bq, bk, bv, bo, ws, &bo_eff, st,

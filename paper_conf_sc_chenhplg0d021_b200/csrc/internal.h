@@ -57,6 +57,8 @@ struct GemmSegment {
   const void* values;       // packed tiles
   const void* bias;         // [seg_rows] in dtype, or nullptr
   int tile_rows;            // number of 16-row tile rows in this segment
+  int rp_stride;            // row_ptr entries between K parts (0: tile_rows + 1; a row slice of a larger
+                            // packed weight passes row_ptr + first row and the weight's tile rows + 1)
   int out_col;              // first output column of the segment in Y
   float scale;              // epilogue scale for ET_EPI_BIAS_SCALE (applied if apply_scale)
   int apply_scale;
@@ -143,6 +145,7 @@ struct VPrep {
   const void* bv;
   const void* bo;
   int heads, d_k;
+  int f_begin, f_end;  // pruned V features folded into b_O': f in [f_begin, f_end) (the call's heads)
   et_dtype dtype;
   int32_t* v_col;      // out [H]
   int32_t* v_width;    // out [H]

@@ -74,7 +74,7 @@ __global__ void vprep_bias_kernel(const int32_t* __restrict__ row_map, int rows_
 // was the longest kernel of a C2 forward: 27 us on 4 SMs.)
 __global__ void vprep_fold_kernel(const uint8_t* __restrict__ wo_values, const int32_t* __restrict__ wo_prp,
                                   const int32_t* __restrict__ wo_tile_col, int wo_tile_rows, int kparts,
-                                  const uint32_t* __restrict__ wv_mask, const void* __restrict__ bv,
+                                  const uint32_t* __restrict__ wv_mask, int f0, int f1, const void* __restrict__ bv,
                                   const void* __restrict__ bo, et_dtype dt, int d, void* __restrict__ bo_folded) {
   const int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
@@ -87,7 +87,7 @@ __global__ void vprep_fold_kernel(const uint8_t* __restrict__ wo_values, const i
     for (int e = lane; e < ne; e += 32) {
       const int t = t0 + (e >> 4), k = e & 15;
       const int f = wo_tile_col[t] * 16 + k;
-      if ((wv_mask[f >> 5] >> (f & 31)) & 1u) continue;   // kept V feature: no fold
+      if (f < f0 || f >= f1 || ((wv_mask[f >> 5] >> (f & 31)) & 1u)) continue;   // kept / other heads: no fold
       const uint8_t* tile = wo_values + (size_t)t * 256 * (dt == ET_FP32 ? 4 : 2);
       float w;
       if (dt == ET_FP32) {   // FP32 tiles: row-major (simt32.cu)
@@ -133,7 +133,8 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream) {
   const int d = v.wo->rows;
   vprep_fold_kernel<<<(d + 3) / 4, 128, 0, stream>>>(static_cast<const uint8_t*>(v.wo->values),
                                                          v.wo->part_row_ptr, v.wo->tile_col, v.wo->rows / 16,
-                                                         v.wo->kparts, v.wv->mask, v.bv, v.bo, v.dtype, d,
+                                                         v.wo->kparts, v.wv->mask, v.f_begin, v.f_end, v.bv, v.bo,
+                                                         v.dtype, d,
                                                          v.bo_folded);
   count_launch();
   ET_CUDA(cudaGetLastError());

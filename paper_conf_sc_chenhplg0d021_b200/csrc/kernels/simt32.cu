@@ -34,7 +34,7 @@ struct G32Params {
   const int32_t* tile_col[3];
   const float* values[3];
   const float* bias[3];
-  int tile_rows[3], out_col[3];
+  int tile_rows[3], rp_stride[3], out_col[3];
   float scale[3];
   int apply_scale[3];
   float* Y;
@@ -56,7 +56,7 @@ __global__ void __launch_bounds__(256) gemm32_kernel(const G32Params p) {
   const int i = gr - p.row_begin[s];
   const int m0 = blockIdx.y * kTok, z = blockIdx.z;
   const int n = threadIdx.x & 15, tg = threadIdx.x >> 4;   // feature n, tokens tg*4 .. tg*4+3
-  const int32_t* rp = p.prp[s] + (size_t)z * (p.tile_rows[s] + 1);
+  const int32_t* rp = p.prp[s] + (size_t)z * p.rp_stride[s];
   float acc[4] = {0.f, 0.f, 0.f, 0.f};
   for (int t = rp[i]; t < rp[i + 1]; ++t) {
     const int j = p.tile_col[s][t];                        // global tile column (K part z's range)
@@ -192,6 +192,7 @@ et_status gemm32_run(const GemmArgs& a, cudaStream_t stream) {
     p.values[s] = static_cast<const float*>(a.seg[s].values);
     p.bias[s] = static_cast<const float*>(a.seg[s].bias);
     p.tile_rows[s] = a.seg[s].tile_rows;
+    p.rp_stride[s] = a.seg[s].rp_stride ? a.seg[s].rp_stride : a.seg[s].tile_rows + 1;
     p.out_col[s] = a.seg[s].out_col;
     p.scale[s] = a.seg[s].scale;
     p.apply_scale[s] = a.seg[s].apply_scale;

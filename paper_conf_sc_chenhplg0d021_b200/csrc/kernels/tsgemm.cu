@@ -104,11 +104,11 @@ template <int kEpi> struct Roles {
 };
 
 struct SegDev {
-  const int32_t* prp;       // part_row_ptr [kparts][tile_rows + 1]
+  const int32_t* prp;       // part_row_ptr [kparts][rp_stride] (+ the segment's first row)
   const int32_t* tile_col;  // values order
   const uint8_t* values;
   const void* bias;
-  int tile_rows;
+  int tile_rows, rp_stride;
   int out_col;
   float scale;
   int apply_scale;
@@ -238,8 +238,8 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   const int z = blockIdx.z;
   const int nk = min(p.Kp, p.K - z * p.Kp) / 64;   // A chunks (64 K each) of this K part
   const int rowsA = (two ? sa.tile_rows : pc.i1) - pc.i0, rowsB = two ? pc.i1 : 0;
-  const int32_t* rpa = sa.prp + (size_t)z * (sa.tile_rows + 1);
-  const int32_t* rpb = sb.prp + (size_t)z * (sb.tile_rows + 1);
+  const int32_t* rpa = sa.prp + (size_t)z * sa.rp_stride;
+  const int32_t* rpb = sb.prp + (size_t)z * sb.rp_stride;
   const int pbA = rpa[pc.i0], peA = rpa[pc.i0 + rowsA];     // part A's packed tiles [pbA, peA)
   const int pbB = two ? rpb[0] : 0, peB = two ? rpb[rowsB] : 0;
   const int nchA = (peA - pbA + kChunkTiles - 1) / kChunkTiles;   // part B starts on a fresh tile chunk
@@ -320,6 +320,7 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
         const uint4 u = *reinterpret_cast<const uint4*>(rowp + ((c ^ (rr & 7)) << 4));
         v[4 * c] = u.x; v[4 * c + 1] = u.y; v[4 * c + 2] = u.z; v[4 * c + 3] = u.w;
       }
+      fence_proxy_async_smem();   // these generic-proxy reads precede the async-proxy refill of the slot
       __syncwarp();
       if (lane == 0) mbar_arrive(&bar.xfree[sq]);   // the producer may reuse the slot
       tmem_st32(tq + j * 32, v);
@@ -896,6 +897,7 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     prm.seg[s].values = static_cast<const uint8_t*>(gs.values);
     prm.seg[s].bias = gs.bias;
     prm.seg[s].tile_rows = gs.tile_rows;
+    prm.seg[s].rp_stride = gs.rp_stride ? gs.rp_stride : gs.tile_rows + 1;
     prm.seg[s].out_col = gs.out_col;
     prm.seg[s].scale = gs.scale;
     prm.seg[s].apply_scale = gs.apply_scale;

@@ -153,19 +153,23 @@ def pack_head_slice(raw: dict, full, heads: int, h0: int, h1: int, dtype="fp16")
 class HeadParallelEncoder:
     """Post-LN encoder stack in head-parallel mode on this rank (one process per GPU).
 
-    Per layer: et_attention_fwd on the rank's head slice -> FP32 partial [M, d] -> all-reduce(sum)
-    over `group` (skipped at world size 1) -> et_layernorm_fwd (residual + LN, Y1) -> FFN1 / FFN2
-    (et_linear_fwd, replicated on every rank) -> et_layernorm_fwd (Y2).  Every rank processes the
-    whole batch; the outputs are identical on all ranks.  Residual stream in the operand dtype."""
+    Per layer: et_attention_fwd on the FULL packed weights with the rank's head range (the library
+    slices them) -> FP32 partial [M, d] -> all-reduce(sum) over `group` (skipped at
+    world size 1) -> et_layernorm_fwd (residual + LN, Y1) -> FFN1 / FFN2 (et_linear_fwd, replicated on
+    every rank) -> et_layernorm_fwd (Y2).  Every rank processes the whole batch; the outputs are
+    identical on all ranks.  Residual stream in the operand dtype.  `capture()` records the whole
+    forward, NCCL all-reduces included, as one CUDA graph (torch.cuda.graph on the current stream).
+    slices=True: the caller-sliced form instead (dist.pack_head_slice re-packs each rank's slices)."""
 
     def __init__(self, raws: list, full_layers: list, heads: int, batch: int, seq_len: int, d_ff: int,
                  act="gelu", ln_eps=1e-12, dtype="fp16", causal=False, mode="auto", lengths=None,
-                 rank: int = 0, world: int = 1, group=None):
+                 rank: int = 0, world: int = 1, group=None, slices: bool = False):
         import paper_conf_sc_chenhplg0d021_b200 as et
         self.et = et
         self.h0, self.h1 = head_range(heads, world, rank)
         self.full = full_layers
-        self.slices = [pack_head_slice(r, f, heads, self.h0, self.h1, dtype) for r, f in zip(raws, full_layers)]
+        self.slices = ([pack_head_slice(r, f, heads, self.h0, self.h1, dtype) for r, f in zip(raws, full_layers)]
+                       if slices else list(full_layers))
         self.heads, self.batch, self.seq_len, self.d_ff = heads, batch, seq_len, d_ff
         self.act_epi = et.EPI_BIAS_GELU if act == "gelu" else et.EPI_BIAS_RELU
         self.eps, self.dtype, self.causal, self.mode, self.lengths = ln_eps, dtype, causal, mode, lengths
@@ -208,11 +212,28 @@ class HeadParallelEncoder:
         et.layernorm_fwd(self.p2, D["b2"], self.y1, D["ln2_g"], D["ln2_b"], self.eps, self.dtype, self.dtype,
                          out_act=dst)
 
+    def capture(self, X: torch.Tensor, out: torch.Tensor):
+        """The whole forward on (X, out) as one CUDA graph, the per-layer NCCL all-reduce included
+        (torch captures NCCL collectives on the capture stream); replay with g.replay()."""
+        self._tmp = torch.empty_like(X) if len(self.full) > 1 else None
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):   # warm-up on a side stream (NCCL communicator init, lazy state)
+            self(X, out)
+        torch.cuda.current_stream().wait_stream(s)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            self(X, out)
+        return g
+
     def __call__(self, X: torch.Tensor, out: torch.Tensor | None = None) -> torch.Tensor:
         cur = X
         if out is None:
             out = torch.empty_like(X)
-        tmp = torch.empty_like(X) if len(self.full) > 1 else None
+        tmp = getattr(self, "_tmp", None)
+        if tmp is None and len(self.full) > 1:
+            tmp = self._tmp = torch.empty_like(X)
         for l in range(len(self.full)):
             part = self.attn_partial(l, cur)
             self._allreduce(part)                                   # NCCL over NVLink on GPUs

@@ -62,6 +62,41 @@ def test_head_parallel_partials_sum_to_full_block(etm, key, kw, worlds):
         assert_close(to64(total), to64(whole), max_abs=1e-2, rel_fro=2e-3, what=f"{key} world {world} vs full call")
 
 
+@pytest.mark.parametrize("key,kw,worlds", [
+    ("C3", {"layers": 1, "batch": 2}, (2, 3, 8)),
+    ("C2", {}, (2, 4)),
+    ("C3", {"layers": 1, "batch": 2, "dtype": "bf16"}, (2,)),
+    ("C4", {"layers": 1, "batch": 1, "seq_len": 384}, (3,)),
+])
+def test_head_range_on_full_weights(etm, key, kw, worlds):
+    """et_attention_fwd with the FULL packed weights and [head_begin, head_end): the
+    library slices W_Q / W_K / W_V by tile rows (a row-pruned W_V is projected whole), runs W_O over a
+    full-width Z that is zero outside the range, and folds only the range's pruned-V bias.  The ranks'
+    partials sum to the oracle's block and agree with the caller-sliced partials."""
+    from paper_conf_sc_chenhplg0d021_b200.dist import head_range, pack_head_slice
+    cfg, raws, X, lens = _case(key, **kw)
+    raw = raws[0]
+    full = etm.pack_layer(raw, cfg.scheme, cfg.ratio, cfg.heads, cfg.dtype)
+    L = torch.from_numpy(lens).cuda()
+    Xd = dev_tensor(X.reshape(cfg.tokens, cfg.d_model), cfg.dtype)
+    w = oe.prune_layer(raw, cfg.scheme, cfg.ratio)[0]
+    ref = oe.attention_block(X.astype(np.float64), w, cfg.heads, lens, cfg.causal).reshape(cfg.tokens, cfg.d_model)
+    for world in worlds:
+        parts = []
+        for r in range(world):
+            h0, h1 = head_range(cfg.heads, world, r)
+            p = etm.attention_fwd(Xd, full, cfg.batch, cfg.seq_len, cfg.heads, L, cfg.causal, ln=False,
+                                  head_range=(h0, h1))
+            sl = etm.attention_fwd(Xd, pack_head_slice(raw, full, cfg.heads, h0, h1, cfg.dtype), cfg.batch,
+                                   cfg.seq_len, cfg.heads, L, cfg.causal, ln=False, head_range=(h0, h1))
+            torch.cuda.synchronize()
+            assert_close(to64(p), to64(sl), max_abs=2e-3, rel_fro=1e-3, what=f"{key} rank {r}/{world} full vs slices")
+            parts.append(p)
+        total = torch.stack(parts).sum(0)
+        torch.cuda.synchronize()
+        assert_close(to64(total), ref, what=f"{key} world {world} (full weights) vs oracle")
+
+
 def test_head_slice_masks_match_full_pack(etm):
     """The slices keep exactly the full matrices' tiles (bit-exact, unpacked values included)."""
     from paper_conf_sc_chenhplg0d021_b200.dist import pack_head_slice
@@ -83,8 +118,9 @@ def test_head_parallel_rejects_bad_slices(etm):
     with pytest.raises(etm.EtError):       # slice of 4 heads passed as a 6-head range
         etm.attention_fwd(Xd, s, cfg.batch, cfg.seq_len, cfg.heads, ln=False, head_range=(0, 6),
                           out=torch.empty(cfg.tokens, cfg.d_model, device="cuda"))
-    with pytest.raises(etm.EtError):       # full weights with a sub-range
-        etm.attention_fwd(Xd, full, cfg.batch, cfg.seq_len, cfg.heads, ln=False, head_range=(0, 4),
+    mixed = etm.Layer(dict(full.packed, wo=s.packed["wo"]), full.dense)   # full W_Q/K/V with a sliced W_O
+    with pytest.raises(etm.EtError):
+        etm.attention_fwd(Xd, mixed, cfg.batch, cfg.seq_len, cfg.heads, ln=False, head_range=(0, 4),
                           out=torch.empty(cfg.tokens, cfg.d_model, device="cuda"))
 
 
