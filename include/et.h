@@ -212,6 +212,26 @@ et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld
                            int32_t v_off, const int32_t* v_col, const int32_t* v_width, int32_t v_width_max,
                            float scale, void* Z, int32_t ld_z, const int32_t* z_map, void* stream);
 
+/* Paper-literal partial on-the-fly attention (§3.2 "partial OTF", Fig. 8 line
+ * 236; the switch at sequence length 224, line 244) — the design the fused short / long forms of
+ * et_attn_core_fwd replace, kept to measure that trade-off on B200:
+ *   kernel A   S_h = Q_h . K_h^T for h in [head_begin, head_end), written to `scores` as 16-bit
+ *              (desc->dtype; the paper's pure FP16, line 157-159 — pass Q pre-scaled by 1/sqrt(d_k));
+ *   kernel B   per query row i: mask (keys j >= len_b; j > i if causal), softmax(scale * S_h[i, :])
+ *              two-pass exact over the stored row, P rounded to 16 bit, Z_h[i] = (P . V_h) / rowsum.
+ * qkv, q_off, k_off, v_off, Z, ld_z: as et_attn_core_fwd with dense V (v_col = v_width = z_map = NULL):
+ * head h reads columns q_off + h*d_k ..., writes Z columns (h - head_begin)*d_k ....
+ * Requirements: dtype FP16 / BF16, d_k 64 or 128, seq_len % 8 == 0, 16-byte aligned qkv / Z rows
+ * (ET_ERR_UNSUPPORTED / ET_ERR_INVALID_ARG otherwise).
+ * scores: caller-owned device buffer of et_attn_partial_scores_bytes() bytes, 16-byte aligned,
+ * layout [batch][head_end - head_begin][seq_len][round_up(seq_len, 8)] 16-bit; score blocks of keys
+ * >= len_b (and above the diagonal when causal) are not written.  ET_ERR_WORKSPACE if too small.
+ * Two launches on `stream`, graph capturable, no allocation. */
+et_status et_attn_partial_scores_bytes(const et_attn_desc* desc, size_t* bytes);
+et_status et_attn_partial_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld_qkv, int32_t q_off,
+                              int32_t k_off, int32_t v_off, float scale, void* Z, int32_t ld_z, void* scores,
+                              size_t scores_bytes, void* stream);
+
 /* Self-attention block (Fig. 3(a) steps 1-7, Eq. 3-4):
  *   out = SelfAttn(X)                  if ln_gamma == NULL
  *   out = LN(X + SelfAttn(X))          otherwise (post-LN, line 75)
@@ -220,12 +240,17 @@ et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld
  *
  * Head-parallel mode (desc->head_begin/head_end = [h0, h1) != [0, H); Megatron-style split of
  * Eq. 4: Output = sum_h Z_h . W_O,h^T, so each rank computes the sum over its heads and
- * an all-reduce(sum) over ranks gives the full output):
- *   wq, wk, wv  the rank's ROW slices [(h1-h0)*d_k, d_model] of the full matrices (rows h0*d_k ..),
- *   wo          its COLUMN slice [d_model, (h1-h0)*d_k] (columns h0*d_k ..),
- *               each packed with mask_in = the full matrix's mask restricted to the slice, so the
- *               kept set is the one the whole-matrix ranking chose (pruning is per matrix, C-3);
- *   bq, bk, bv  the matching slices of the biases; bo the full [d_model] bias;
+ * an all-reduce(sum) over ranks gives the full output).  The weights are either
+ *   (a) the FULL packed matrices (wq->rows == d_model): the library projects only the range's tile
+ *       rows of W_Q / W_K / W_V (a ROW-pruned W_V is projected whole; its per-head packed windows
+ *       are located on the device) and runs W_O over a full-width Z that is zero outside the range;
+ *       h0*d_k and (h1-h0)*d_k must be multiples of 16 (ET_ERR_UNSUPPORTED otherwise); or
+ *   (b) the caller's slices: wq, wk, wv the rank's ROW slices [(h1-h0)*d_k, d_model] of the full
+ *       matrices (rows h0*d_k ..), wo its COLUMN slice [d_model, (h1-h0)*d_k] (columns h0*d_k ..),
+ *       each packed with mask_in = the full matrix's mask restricted to the slice, so the kept set
+ *       is the one the whole-matrix ranking chose (pruning is per matrix, C-3); bq, bk, bv the
+ *       matching slices of the biases;
+ *   bo          the full [d_model] bias in both cases;
  *   ln_gamma    must be NULL (residual + LN follow the all-reduce: et_layernorm_fwd);
  *   out         FP32 [batch*seq_len, d_model] (reading C-21: FP32 partials) =
  *               sum_{h in [h0,h1)} Z_h W_O,h^T  + b_O (only if h0 == 0)
@@ -250,8 +275,9 @@ typedef struct {
  * X, out: [batch*seq_len, d_model] in resid_dtype (FP32, or equal to desc->dtype; reading C-22);
  * GEMM operands in desc->dtype.  layers_host: host array of num_layers et_layer.  X and out
  * may alias.  No host synchronisation; CUDA-graph capturable.  Full head range only
- * (ET_ERR_UNSUPPORTED otherwise): a head-parallel layer is et_attention_fwd on the rank's slices,
- * an all-reduce of the FP32 partials by the caller's process group, then et_layernorm_fwd. */
+ * (ET_ERR_UNSUPPORTED otherwise): a head-parallel layer is et_attention_fwd on the rank's head range
+ * (full weights or the rank's slices), an all-reduce of the FP32 partials by the caller's process
+ * group, then et_layernorm_fwd. */
 et_status et_encoder_workspace_size(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff,
                                     et_dtype resid_dtype, const et_layer* layers_host, size_t* bytes);
 et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff, et_act act, float ln_eps,

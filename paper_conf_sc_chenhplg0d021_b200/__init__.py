@@ -325,6 +325,35 @@ def attn_core_fwd(qkv: torch.Tensor, batch: int, seq_len: int, heads: int, d_mod
     return Z
 
 
+_partial_bytes = _sig("et_attn_partial_scores_bytes", ctypes.c_int, [ctypes.POINTER(AttnDescC), ctypes.POINTER(_sz)])
+_partial = _sig("et_attn_partial_fwd", ctypes.c_int,
+                [ctypes.POINTER(AttnDescC), _vp, _i32, _i32, _i32, _i32, _f32, _vp, _i32, _vp, _sz, _vp])
+SYMBOLS += ["et_attn_partial_scores_bytes", "et_attn_partial_fwd"]
+
+
+def attn_partial_scores_bytes(batch: int, seq_len: int, heads: int, d_model: int, dtype="fp16",
+                              head_begin: int = 0, head_end: int | None = None) -> int:
+    d = attn_desc(batch, seq_len, heads, d_model, dtype, head_begin=head_begin, head_end=head_end)
+    n = _sz(0)
+    _check(_partial_bytes(ctypes.byref(d), ctypes.byref(n)))
+    return int(n.value)
+
+
+def attn_partial_fwd(qkv: torch.Tensor, batch: int, seq_len: int, heads: int, d_model: int, q_off: int, k_off: int,
+                     v_off: int, lengths=None, causal=False, scale: float = 1.0, Z=None, scores=None, stream=None):
+    """et_attn_partial_fwd: the paper's partial OTF (Fig. 8) — Q.K^T materialised
+    in a 16-bit score buffer, then mask + softmax + x V per row.  Returns (Z, scores)."""
+    d = attn_desc(batch, seq_len, heads, d_model, qkv.dtype, lengths, causal)
+    if Z is None:
+        Z = torch.zeros(batch * seq_len, d_model, dtype=qkv.dtype, device=qkv.device)
+    if scores is None:
+        nbytes = attn_partial_scores_bytes(batch, seq_len, heads, d_model, qkv.dtype)
+        scores = torch.empty(nbytes // 2, dtype=qkv.dtype, device=qkv.device)
+    _check(_partial(ctypes.byref(d), qkv.data_ptr(), qkv.stride(0), q_off, k_off, v_off, scale, Z.data_ptr(),
+                    Z.stride(0), scores.data_ptr(), scores.numel() * scores.element_size(), _stream(stream)))
+    return Z, scores
+
+
 # ------------------------------------------------------------------------------------------ layers
 class Layer:
     """One packed encoder layer: six packed weights + device biases / LayerNorm parameters."""

@@ -313,6 +313,41 @@ et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld
   return attention_run(a, static_cast<cudaStream_t>(stream));
 }
 
+et_status et_attn_partial_scores_bytes(const et_attn_desc* desc, size_t* bytes) {
+  ET_TRY(check_desc(desc));
+  if (!bytes) return fail(ET_ERR_INVALID_ARG, "et_attn_partial_scores_bytes: null pointer");
+  *bytes = attention_partial_scores_bytes(desc->batch, desc->seq_len, desc->head_end - desc->head_begin);
+  return ET_OK;
+}
+
+et_status et_attn_partial_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld_qkv, int32_t q_off,
+                              int32_t k_off, int32_t v_off, float scale, void* Z, int32_t ld_z, void* scores,
+                              size_t scores_bytes, void* stream) {
+  ET_TRY(check_desc(desc));
+  if (!qkv || !Z || !scores) return fail(ET_ERR_INVALID_ARG, "et_attn_partial_fwd: null pointer");
+  AttnArgs a{};
+  a.qkv = qkv;
+  a.ld_qkv = ld_qkv;
+  a.q_off = q_off;
+  a.k_off = k_off;
+  a.v_off = v_off;
+  a.Z = Z;
+  a.ld_z = ld_z;
+  a.lengths = desc->lengths_dev;
+  a.batch = desc->batch;
+  a.seq_len = desc->seq_len;
+  a.heads = desc->heads;
+  a.d_k = desc->d_model / desc->heads;
+  a.head_begin = desc->head_begin;
+  a.head_end = desc->head_end;
+  a.causal = desc->causal;
+  a.v_width_max = a.d_k;
+  a.scale = scale;
+  a.dtype = desc->dtype;
+  a.ts = trace_slot(ET_K_ATTN);
+  return attention_partial_run(a, scores, scores_bytes, static_cast<cudaStream_t>(stream));
+}
+
 et_status et_attention_workspace_size(const et_attn_desc* desc, const et_packed_weight* wv, size_t* bytes) {
   ET_TRY(check_desc(desc));
   if (!wv || !bytes) return fail(ET_ERR_INVALID_ARG, "et_attention_workspace_size: null pointer");

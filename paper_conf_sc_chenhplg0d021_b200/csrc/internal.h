@@ -134,6 +134,10 @@ et_status attention32_run(const AttnArgs& a, cudaStream_t stream);
 bool attention128_applies(const AttnArgs& a);
 et_status attention128_run(const AttnArgs& a, cudaStream_t stream);
 int attn_short_max(int d_k);
+// paper-literal partial OTF (kernels/attention_partial.cu): S = Q K^T materialised in 16 bit,
+// then mask + softmax + x V per row
+size_t attention_partial_scores_bytes(int batch, int seq_len, int heads);
+et_status attention_partial_run(const AttnArgs& a, void* scores, size_t scores_bytes, cudaStream_t stream);
 
 // ---------------------------------------------------------------- small helpers (kernels/layernorm.cu)
 et_status cast_run(const void* src, et_dtype sdt, void* dst, et_dtype ddt, size_t n, cudaStream_t stream);

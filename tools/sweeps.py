@@ -1,8 +1,9 @@
 """SURVEY §8(d) diagnostics beside the headline (run on the GPU box; JSON lines to stdout):
   M2  sparsity sweep (Fig. 10 / line 252 analogue): the tile-sparse linear layer at M = 4096
       tokens for d x d (d = 768, 1024) and the BERT FFN shapes, tile ratio 0 ... 0.95;
-  M3  sequence-length crossover (Fig. 8 / line 244 analogue): short vs long attention form at fixed
-      total tokens, BERT-base heads (H = 12, d_k = 64).
+  M3  sequence-length crossover (Fig. 8 / line 244 analogue): short vs long attention form vs the
+      paper-literal partial OTF at fixed total tokens, BERT-base heads (H = 12, d_k = 64);
+  M3b the same at batch 1 (Fig. 8's setting), BERT-base and Transformer heads.
 Timing: CUDA events around 50 back-to-back launches after 5 warm-ups (operands L2-resident when they
 fit: a kernel-level diagnostic, not the bench metric).  Dense torch.matmul at the same shape is
 printed as context only (it is never a backend)."""
@@ -105,29 +106,54 @@ def m2b():
             print(json.dumps(row), flush=True)
 
 
-def m3():
-    H, dk, total = 12, 64, 32768
+def _m3_row(tag, S, B, H, dk):
     d = H * dk
+    qkv = (torch.randn(B * S, 3 * d, device="cuda") * 0.5).half()
+    Z = torch.empty(B * S, d, device="cuda").half()
+    scores = torch.empty(et.attn_partial_scores_bytes(B, S, H, d, "fp16") // 2, dtype=torch.float16, device="cuda")
+    flops = 4.0 * B * H * S * S * dk
+    row = {"sweep": tag, "S": S, "B": B, "H": H, "d_k": dk}
+    for mode in ("short", "long", "partial"):
+        if mode == "short" and S > et.attn_short_max(dk):
+            continue
+        if mode == "partial":
+            fn = lambda: et.attn_partial_fwd(qkv, B, S, H, d, 0, d, 2 * d, Z=Z, scores=scores)
+        else:
+            fn = lambda: et.attn_core_fwd(qkv, B, S, H, d, 0, d, 2 * d, mode=mode, scale=1.0, Z=Z)
+        us = timed(fn)
+        row[f"{mode}_us"] = round(us, 2)
+        row[f"{mode}_eff_tflops"] = round(flops / us / 1e6, 1)
+    fused = min(v for k, v in row.items() if k in ("short_us", "long_us"))
+    row["partial_over_fused"] = round(row["partial_us"] / fused, 2)
+    # the partial form's extra HBM traffic: the 16-bit score matrix written once, read twice
+    row["partial_score_bytes"] = int(3 * B * H * S * S * 2)
+    print(json.dumps(row), flush=True)
+
+
+def m3():
+    """Fixed total tokens (32768), BERT-base heads: the fused short / long forms vs the paper-literal
+    partial OTF (et_attn_partial_fwd, NEXT-2)."""
+    H, dk, total = 12, 64, 32768
     for S in (64, 128, 192, 224, 256, 320, 384, 512, 1024, 2048):
-        B = max(1, total // S)
-        qkv = torch.randn(B * S, 3 * d, device="cuda").half()
-        Z = torch.empty(B * S, d, device="cuda").half()
-        flops = 4.0 * B * H * S * S * dk
-        row = {"sweep": "M3", "S": S, "B": B, "H": H, "d_k": dk}
-        for mode in ("short", "long"):
-            if mode == "short" and S > et.attn_short_max(dk):
-                continue
-            us = timed(lambda: et.attn_core_fwd(qkv, B, S, H, d, 0, d, 2 * d, mode=mode, scale=0.125, Z=Z))
-            row[f"{mode}_us"] = round(us, 2)
-            row[f"{mode}_eff_tflops"] = round(flops / us / 1e6, 1)
-        print(json.dumps(row), flush=True)
+        _m3_row("M3", S, max(1, total // S), H, dk)
+
+
+def m3b():
+    """Fig. 8's own setting: one sequence, BERT-base (H = 12) and the
+    Transformer (d_model 512, H = 8), S = 64 ... 2048 — latency-bound; where the paper's full OTF
+    vs partial OTF crossover (224 on V100S) lands on B200."""
+    for H in (12, 8):
+        for S in (64, 128, 192, 224, 256, 320, 384, 512, 768, 1024, 2048):
+            _m3_row("M3b", S, 1, H, 64)
 
 
 if __name__ == "__main__":
-    which = sys.argv[1:] or ["m2", "m2b", "m3"]
+    which = sys.argv[1:] or ["m2", "m2b", "m3", "m3b"]
     if "m2" in which:
         m2()
     if "m2b" in which:
         m2b()
     if "m3" in which:
         m3()
+    if "m3b" in which:
+        m3b()
