@@ -27,6 +27,8 @@ namespace et {
 
 et_status make_tmap_2d(CUtensorMap* tm, const void* base, et_dtype dtype, uint64_t rows, uint64_t cols,
                        uint64_t ld_elems, uint32_t box_cols, uint32_t box_rows, bool swizzle128);
+et_status make_tmap_3d_ld(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t cols, uint64_t rows, uint64_t planes,
+                          uint64_t ld_elems, uint32_t box_cols, uint32_t box_rows);
 
 namespace {
 
@@ -34,8 +36,7 @@ struct PParams {
   int S, H, head_begin, nh;   // nh = heads in the call
   int q_off, k_off, v_off;
   const int32_t* lengths;
-  uint16_t* scores;           // [B * nh][S][ld_s] 16-bit
-  int ld_s;
+  int ld_s;                   // row pitch of the [B * nh][S][ld_s] 16-bit score buffer (tensor map)
   void* Z;
   int ld_z;
   int causal;
@@ -52,103 +53,164 @@ __device__ __forceinline__ float ex2p(float x) {
 }
 
 // ----------------------------------------------------------------- kernel A: S = Q~ K^T to global
+// One CTA per (128-query block, batch x head): Q resident in shared memory, K blocks of 128 keys
+// streamed through a TMA ring, two 128-column TMEM accumulators so the epilogue of key block kb
+// overlaps the MMAs of kb + 1, and the 16-bit score tile leaving through shared memory by TMA
+// store (whole 128-byte lines; rows / keys past seq_len are clipped by the tensor map).
+// warp 0: TMA producer, warp 1: MMA issuer + TMEM owner, warps 2-5: epilogue (TMEM lane quarter w%4).
+template <int kDK> struct QktCfg {
+  static constexpr int kTiles = kDK / 64;               // 64-column SWIZZLE_128B boxes per operand
+  static constexpr int kOpBytes = kTiles * 16384;       // one 128-row Q or K block
+  static constexpr int kKS = kDK == 64 ? 4 : 2;         // K ring stages (one CTA per SM; 2 stages measured slower)
+  static constexpr int kStage = 32768;                  // one 128 x 128 16-bit score tile (two boxes)
+  static constexpr int kSmem = 1024 + kOpBytes * (1 + kKS) + 2 * kStage;
+};
+
 template <bool kBF16, int kDK>
-__global__ void __launch_bounds__(128, 1) qkt_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ PParams p) {
-  constexpr int kTiles = kDK / 64;
+__global__ void __launch_bounds__(192, 1) qkt_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                     const __grid_constant__ CUtensorMap tmap_s,
+                                                     const __grid_constant__ PParams p) {
+  using C = QktCfg<kDK>;
   pdl_trigger();
   pdl_wait();
   trace_cta_start(p.ts);
-  const int qb = blockIdx.x, kb = blockIdx.y, bh = blockIdx.z;
+  const int qb = blockIdx.x, bh = blockIdx.y;
   const int b = bh / p.nh, h = p.head_begin + bh % p.nh;
   const int len = p.lengths ? p.lengths[b] : p.S;
-  // blocks kernel B never reads: keys past the valid length, or above the diagonal when causal
-  if (kb * 128 >= len || (p.causal && kb > qb)) {
-    trace_cta_end(p.ts);
-    return;
-  }
+  // key blocks kernel B reads: keys < len, and <= the block's last query when causal
+  int nkb = (len + 127) / 128;
+  if (p.causal) nkb = min(nkb, qb + 1);
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sQ = smem;
-  uint8_t* sK = smem + kTiles * 16384;
-  __shared__ uint64_t full, done;
+  uint8_t* sK = smem + C::kOpBytes;
+  uint8_t* sO = sK + C::kKS * C::kOpBytes;
+  __shared__ uint64_t q_full, k_full[C::kKS], k_free[C::kKS], acc_full[2], acc_free[2];
   __shared__ uint32_t tslot;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
-    mbar_init(&full, 1);
-    mbar_init(&done, 1);
+    mbar_init(&q_full, 1);
+    for (int i = 0; i < C::kKS; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_free[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&acc_full[i], 1);
+      mbar_init(&acc_free[i], 4);
+    }
     fence_mbar_init();
   }
-  if (warp == 0) tmem_alloc<128>(&tslot);
+  if (warp == 1) tmem_alloc<256>(&tslot);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tb = tslot;
   const int row0 = b * p.S;
+  const uint32_t op_tx = (uint32_t)C::kTiles * p.box_rows * 128;
   if (warp == 0) {
     if (lane == 0) {
-      const uint32_t tile = (uint32_t)p.box_rows * 128;
-      mbar_expect_tx(&full, 2 * kTiles * tile);
-      for (int t = 0; t < kTiles; ++t) {
-        tma_load_2d(sQ + t * 16384, &tmap, &full, p.q_off + h * kDK + t * 64, row0 + qb * 128);
-        tma_load_2d(sK + t * 16384, &tmap, &full, p.k_off + h * kDK + t * 64, row0 + kb * 128);
+      mbar_expect_tx(&q_full, op_tx);
+      for (int t = 0; t < C::kTiles; ++t)
+        tma_load_2d(sQ + t * 16384, &tmap, &q_full, p.q_off + h * kDK + t * 64, row0 + qb * 128);
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int st = kb % C::kKS;
+        if (kb >= C::kKS) mbar_wait(&k_free[st], ((kb / C::kKS) - 1) & 1);
+        mbar_expect_tx(&k_full[st], op_tx);
+        for (int t = 0; t < C::kTiles; ++t)
+          tma_load_2d(sK + st * C::kOpBytes + t * 16384, &tmap, &k_full[st], p.k_off + h * kDK + t * 64,
+                      row0 + kb * 128);
       }
     }
-    mbar_wait_warp(&full, 0);
-    tc_fence_after();
+  } else if (warp == 1) {
     const uint32_t idesc = make_idesc_f16(128, 128, kBF16 ? 1 : 0, 0, 0);
+    mbar_wait_warp(&q_full, 0);
+    for (int kb = 0; kb < nkb; ++kb) {
+      const int st = kb % C::kKS, a = kb & 1;
+      if (kb >= 2) mbar_wait_warp(&acc_free[a], ((kb >> 1) - 1) & 1);
+      mbar_wait_warp(&k_full[st], (kb / C::kKS) & 1);
+      tc_fence_after();
+      const uint32_t qu = smem_u32(sQ), ku = smem_u32(sK + st * C::kOpBytes);
 #pragma unroll
-    for (int ks = 0; ks < kDK / 16; ++ks) {
-      const uint32_t off = (ks >> 2) * 16384 + (ks & 3) * 32;
-      mma_ss_warp(tb, make_sdesc(smem_u32(sQ) + off, 16, 1024, kLayoutSW128),
-                  make_sdesc(smem_u32(sK) + off, 16, 1024, kLayoutSW128), idesc, ks > 0);
+      for (int ks = 0; ks < kDK / 16; ++ks) {
+        const uint32_t off = (ks >> 2) * 16384 + (ks & 3) * 32;
+        mma_ss_warp(tb + a * 128, make_sdesc(qu + off, 16, 1024, kLayoutSW128),
+                    make_sdesc(ku + off, 16, 1024, kLayoutSW128), idesc, ks > 0);
+      }
+      mma_commit_warp(&k_free[st]);
+      mma_commit_warp(&acc_full[a]);
     }
-    mma_commit_warp(&done);
-  }
-  mbar_wait_warp(&done, 0);
-  tc_fence_after();
-  // each thread: its query row's 128 scores -> 16-bit -> global (256 contiguous bytes per row)
-  const int qi = qb * 128 + warp * 32 + lane;
-  uint16_t* dst = p.scores + ((size_t)bh * p.S + qi) * p.ld_s + kb * 128;
+  } else {
+    const int q = warp & 3, r = q * 32 + lane;
+    const bool leader = warp == 2 && lane == 0;
+    for (int kb = 0; kb < nkb; ++kb) {
+      const int a = kb & 1;
+      uint8_t* stg = sO + a * C::kStage;
+      if (leader) bulk_wait_group_read<1>();   // the store issued from this buffer two tiles ago has read it
+      named_bar_sync(1, 128);
+      mbar_wait(&acc_full[a], (kb >> 1) & 1);
+      tc_fence_after();
 #pragma unroll
-  for (int c = 0; c < 4; ++c) {
-    uint32_t v[32];
-    tmem_ld32(tb + ((uint32_t)(warp * 32) << 16) + c * 32, v);
-    tmem_ld_wait();
-    if (qi < p.S) {
+      for (int c = 0; c < 4; ++c) {
+        uint32_t v[32];
+        tmem_ld32(tb + a * 128 + ((uint32_t)(q * 32) << 16) + c * 32, v);
+        tmem_ld_wait();
+        uint8_t* rowp = stg + (c >> 1) * 16384 + r * 128;
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int k = kb * 128 + c * 32 + u * 8;
-        if (k < p.S)   // S % 8 == 0: whole 16-byte groups
-          *reinterpret_cast<uint4*>(dst + c * 32 + u * 8) =
+        for (int u = 0; u < 4; ++u) {
+          const int unit = (c & 1) * 4 + u;
+          *reinterpret_cast<uint4*>(rowp + ((unit ^ (r & 7)) << 4)) =
               make_uint4(pack2<kBF16>(__uint_as_float(v[8 * u]), __uint_as_float(v[8 * u + 1])),
                          pack2<kBF16>(__uint_as_float(v[8 * u + 2]), __uint_as_float(v[8 * u + 3])),
                          pack2<kBF16>(__uint_as_float(v[8 * u + 4]), __uint_as_float(v[8 * u + 5])),
                          pack2<kBF16>(__uint_as_float(v[8 * u + 6]), __uint_as_float(v[8 * u + 7])));
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&acc_free[a]);
+      fence_proxy_async_smem();
+      named_bar_sync(1, 128);
+      if (leader) {
+        tma_store_3d(&tmap_s, stg, kb * 128, qb * 128, bh);
+        tma_store_3d(&tmap_s, stg + 16384, kb * 128 + 64, qb * 128, bh);
+        bulk_commit_group();
       }
     }
+    if (leader) bulk_wait_group<0>();
   }
   tc_fence_before();
   __syncthreads();
   trace_cta_end(p.ts);
-  if (warp == 0) tmem_dealloc<128>(tb);
+  if (warp == 1) tmem_dealloc<256>(tb);
 }
 
 // ----------------------------------------------------------------- kernel B: mask, softmax, x V
-// warps 0-3: one query row per thread (TMEM lane = row); warp 4: MMA issuer + TMEM owner; warp 5:
-// TMA producer of the V blocks.  64-key blocks, P and V double-buffered.
+// One CTA per (128-query block, batch x head).  The block's score rows stream through a TMA ring of
+// 128 x 64-key tiles twice: pass 0 takes the row maxima, pass 1 (key blocks in reverse) turns each tile into P = exp(S - max)
+// IN PLACE (same SWIZZLE_128B layout: the tile is then the K-major A operand) and the MMA warp
+// accumulates P . V_block into TMEM.  The second pass hits L2 (a CTA's rows: 128 x seq_len x 2 B).
+// warps 0-3: one query row per thread (TMEM lane = row); warp 4: MMA issuer + TMEM owner + releaser
+// of pass-0 tiles; warp 5: TMA producer (score tiles, and in pass 1 the V blocks).
+template <int kDK> struct PvCfg {
+  static constexpr int kSS = 3;                       // score ring stages (16 KB each; d_k 64: 3 CTAs per SM)
+  static constexpr int kVT = kDK / 64;                // 64-wide column tiles of a V block
+  static constexpr int kVBytes = kVT * 64 * 128;      // 64 keys x d_k 16-bit (MN-major, SWIZZLE_128B)
+  static constexpr int kSmem = 1024 + kSS * 16384 + 2 * kVBytes;
+};
+
 template <bool kBF16, int kDK>
-__global__ void __launch_bounds__(192, 1) softmax_pv_kernel(const __grid_constant__ CUtensorMap tmap_v,
+__global__ void __launch_bounds__(192, 1) softmax_pv_kernel(const __grid_constant__ CUtensorMap tmap_s,
+                                                            const __grid_constant__ CUtensorMap tmap_v,
                                                             const __grid_constant__ PParams p) {
-  constexpr int kVT = kDK / 64;              // 64-wide column tiles of a V block
-  constexpr int kVBytes = kVT * 64 * 128;    // 64 keys x d_k 16-bit (MN-major, SWIZZLE_128B)
+  using C = PvCfg<kDK>;
   pdl_trigger();
   pdl_wait();
   trace_cta_start(p.ts);
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint8_t* sP = smem;                        // 2 x 16 KB: 128 rows x 64 keys, K-major SWIZZLE_128B
-  uint8_t* sV = smem + 2 * 16384;            // 2 x kVBytes
-  __shared__ uint64_t p_full[2], p_free[2], v_full[2], v_free[2], o_full;
+  uint8_t* sS = smem;                        // kSS x (128 rows x 64 keys), K-major SWIZZLE_128B
+  uint8_t* sV = smem + C::kSS * 16384;       // 2 x kVBytes
+  __shared__ uint64_t s_full[C::kSS], s_free[C::kSS], p_full[C::kSS], v_full[2], v_free[2], o_full;
   __shared__ uint32_t tslot;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int qb = blockIdx.x, bh = blockIdx.y;
@@ -160,9 +222,12 @@ __global__ void __launch_bounds__(192, 1) softmax_pv_kernel(const __grid_constan
   const int nkb = (kmax + 63) / 64;
   const int row0 = b * S;
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < C::kSS; ++i) {
+      mbar_init(&s_full[i], 1);
+      mbar_init(&s_free[i], 1);
       mbar_init(&p_full[i], 4);
-      mbar_init(&p_free[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
       mbar_init(&v_full[i], 1);
       mbar_init(&v_free[i], 1);
     }
@@ -173,7 +238,7 @@ __global__ void __launch_bounds__(192, 1) softmax_pv_kernel(const __grid_constan
   if (p.vbox_rows < 64) {
     // fewer than 64 tokens in the whole batch (one key block): the V rows the box does not cover
     // must be finite zeros, not stale shared memory (P is 0 there, but 0 x NaN is NaN)
-    for (int i = threadIdx.x; i < kVBytes / 16; i += blockDim.x)
+    for (int i = threadIdx.x; i < C::kVBytes / 16; i += blockDim.x)
       reinterpret_cast<uint4*>(sV)[i] = make_uint4(0u, 0u, 0u, 0u);
     fence_proxy_async_smem();
   }
@@ -181,75 +246,129 @@ __global__ void __launch_bounds__(192, 1) softmax_pv_kernel(const __grid_constan
   __syncthreads();
   tc_fence_after();
   const uint32_t tb = tslot;
+  const int ni = 2 * nkb;   // pass 0: it = j, pass 1: it = nkb + j
 
   if (warp == 5) {
     if (lane == 0) {
-      const uint32_t box = (uint32_t)p.vbox_rows * 128u;   // 64 keys (fewer if the batch is shorter) x 64 columns
-      for (int j = 0; j < nkb; ++j) {
-        const int st = j & 1;
-        if (j >= 2) mbar_wait(&v_free[st], ((j >> 1) - 1) & 1);
-        mbar_expect_tx(&v_full[st], kVT * box);
-        for (int t = 0; t < kVT; ++t)
-          tma_load_2d(sV + st * kVBytes + t * 8192, &tmap_v, &v_full[st], p.v_off + h * kDK + t * 64, row0 + j * 64);
+      const uint32_t vbox = (uint32_t)p.vbox_rows * 128u;
+      for (int it = 0; it < ni; ++it) {
+        // pass 1 walks the key blocks backwards: the tiles pass 0 read last are still in L2
+        const int st = it % C::kSS, j = it < nkb ? it : ni - 1 - it;
+        if (it >= C::kSS) mbar_wait(&s_free[st], ((it / C::kSS) - 1) & 1);
+        mbar_expect_tx(&s_full[st], 16384u);
+        tma_load_3d(sS + st * 16384, &tmap_s, &s_full[st], j * 64, qb * 128, bh);
+        if (it >= nkb) {
+          const int jj = it - nkb, vs = jj & 1;   // jj: pass-1 step
+          if (jj >= 2) mbar_wait(&v_free[vs], ((jj >> 1) - 1) & 1);
+          mbar_expect_tx(&v_full[vs], C::kVT * vbox);
+          for (int t = 0; t < C::kVT; ++t)
+            tma_load_2d(sV + vs * C::kVBytes + t * 8192, &tmap_v, &v_full[vs], p.v_off + h * kDK + t * 64,
+                        row0 + j * 64);
+        }
       }
     }
   } else if (warp == 4) {
     const uint32_t idesc = make_idesc_f16(128, kDK, kBF16 ? 1 : 0, 0, 1);   // P K-major, V MN-major
-    for (int j = 0; j < nkb; ++j) {
-      const int st = j & 1;
-      mbar_wait_warp(&p_full[st], (j >> 1) & 1);
-      mbar_wait_warp(&v_full[st], (j >> 1) & 1);
+    for (int it = 0; it < ni; ++it) {
+      const int st = it % C::kSS;
+      mbar_wait_warp(&p_full[st], (it / C::kSS) & 1);
+      if (it < nkb) {   // pass 0: the softmax warps have read the tile
+        if (lane == 0) mbar_arrive(&s_free[st]);
+        __syncwarp();
+        continue;
+      }
+      const int j = it - nkb, vs = j & 1;   // pass-1 step (key block nkb - 1 - j)
+      mbar_wait_warp(&v_full[vs], (j >> 1) & 1);
       tc_fence_after();
-      const uint32_t pu = smem_u32(sP + st * 16384), vu = smem_u32(sV + st * kVBytes);
+      const uint32_t pu = smem_u32(sS + st * 16384), vu = smem_u32(sV + vs * C::kVBytes);
 #pragma unroll
       for (int ks = 0; ks < 4; ++ks)   // 64 keys = 4 x K16; V: 16 keys = 16 rows x 128 B = 2048 B
         mma_ss_warp(tb, make_sdesc(pu + ks * 32, 16, 1024, kLayoutSW128),
                     make_sdesc(vu + ks * 2048, 8192, 1024, kLayoutSW128), idesc, (j > 0 || ks > 0) ? 1u : 0u);
-      mma_commit_warp(&p_free[st]);
-      mma_commit_warp(&v_free[st]);
+      mma_commit_warp(&s_free[st]);
+      mma_commit_warp(&v_free[vs]);
     }
     mma_commit_warp(&o_full);
   } else {
     const int r = warp * 32 + lane, qi = qb * 128 + r;
     int kend = len;
     if (p.causal) kend = min(kend, qi + 1);
-    const uint16_t* srow = p.scores + ((size_t)bh * S + min(qi, S - 1)) * p.ld_s;
     const float sl2 = p.scale_log2;
-    // pass 1: row max over the valid keys (stored 16-bit scores, read 8 at a time)
-    float m = -INFINITY;
-    for (int k = 0; k < kend; k += 8) {
-      const uint4 w = __ldg(reinterpret_cast<const uint4*>(srow + k));
-      const uint32_t ww[4] = {w.x, w.y, w.z, w.w};
+    using T2 = typename std::conditional<kBF16, __nv_bfloat162, __half2>::type;
+    // pass 0: row max over the valid keys (packed 16-bit max; masking only in the tile holding kend)
+    T2 m2;
+    {
+      const uint32_t ninf = kBF16 ? 0xFF80FF80u : 0xFC00FC00u;
+      m2 = *reinterpret_cast<const T2*>(&ninf);
+    }
+    for (int j = 0; j < nkb; ++j) {
+      const int it = j, st = it % C::kSS;
+      mbar_wait(&s_full[st], (it / C::kSS) & 1);
+      const uint8_t* rowp = sS + st * 16384 + r * 128;
+      const int k0 = j * 64;
+      if (k0 + 64 <= kend) {
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float2 f = unpack2<kBF16>(ww[i]);
-        if (k + 2 * i < kend) m = fmaxf(m, f.x);
-        if (k + 2 * i + 1 < kend) m = fmaxf(m, f.y);
+        for (int u = 0; u < 8; ++u) {
+          const uint4 w = *reinterpret_cast<const uint4*>(rowp + ((u ^ (r & 7)) << 4));
+          m2 = __hmax2(m2, __hmax2(__hmax2(*reinterpret_cast<const T2*>(&w.x), *reinterpret_cast<const T2*>(&w.y)),
+                                   __hmax2(*reinterpret_cast<const T2*>(&w.z), *reinterpret_cast<const T2*>(&w.w))));
+        }
+      } else if (k0 < kend) {
+        float mf = -INFINITY;
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const uint4 w = *reinterpret_cast<const uint4*>(rowp + ((u ^ (r & 7)) << 4));
+          const uint32_t ww[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float2 f = unpack2<kBF16>(ww[i]);
+            const int k = k0 + u * 8 + 2 * i;
+            if (k < kend) mf = fmaxf(mf, f.x);
+            if (k + 1 < kend) mf = fmaxf(mf, f.y);
+          }
+        }
+        const uint32_t mp = pack2<kBF16>(mf, mf);   // exact: mf is a 16-bit value
+        m2 = __hmax2(m2, *reinterpret_cast<const T2*>(&mp));
       }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&p_full[st]);
+    }
+    float m;
+    {
+      const uint32_t mu = *reinterpret_cast<const uint32_t*>(&m2);
+      const float2 mf = unpack2<kBF16>(mu);
+      m = fmaxf(mf.x, mf.y);
     }
     const float mb = m * sl2;
     float l = 0.f;
-    // pass 2: P = exp(S - max) per 64-key block into the shared-memory A operand
-    for (int j = 0; j < nkb; ++j) {
-      const int st = j & 1;
-      if (j >= 2) mbar_wait(&p_free[st], ((j >> 1) - 1) & 1);
-      uint8_t* prow = sP + st * 16384 + r * 128;
+    // pass 1: P = exp(S - max) in place, 16-bit, K-major A operand of P . V
+    for (int jj = 0; jj < nkb; ++jj) {
+      const int it = nkb + jj, st = it % C::kSS, j = nkb - 1 - jj;
+      mbar_wait(&s_full[st], (it / C::kSS) & 1);
+      uint8_t* rowp = sS + st * 16384 + r * 128;
+      const int k0 = j * 64;
+      const bool full = k0 + 64 <= kend;
 #pragma unroll
       for (int u = 0; u < 8; ++u) {
-        const int k = j * 64 + u * 8;
-        uint4 w = make_uint4(0u, 0u, 0u, 0u);
-        if (k < kend) w = __ldg(reinterpret_cast<const uint4*>(srow + k));
+        uint4* cell = reinterpret_cast<uint4*>(rowp + ((u ^ (r & 7)) << 4));
+        const uint4 w = *cell;
         const uint32_t ww[4] = {w.x, w.y, w.z, w.w};
         uint32_t pk[4];
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           const float2 f = unpack2<kBF16>(ww[i]);
-          const float p0 = k + 2 * i < kend ? ex2p(f.x * sl2 - mb) : 0.f;
-          const float p1 = k + 2 * i + 1 < kend ? ex2p(f.y * sl2 - mb) : 0.f;
-          l += p0 + p1;
+          const int k = k0 + u * 8 + 2 * i;
+          float p0 = ex2p(f.x * sl2 - mb), p1 = ex2p(f.y * sl2 - mb);
+          if (!full) {
+            p0 = k < kend ? p0 : 0.f;
+            p1 = k + 1 < kend ? p1 : 0.f;
+          }
           pk[i] = pack2<kBF16>(p0, p1);
+          // the row sum takes P as rounded, so that Z = (P . V) / l normalises what the MMA used
+          const float2 pr = unpack2<kBF16>(pk[i]);
+          l += pr.x + pr.y;
         }
-        *reinterpret_cast<uint4*>(prow + ((u ^ (r & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        *cell = make_uint4(pk[0], pk[1], pk[2], pk[3]);
       }
       fence_proxy_async_smem();
       __syncwarp();
@@ -258,7 +377,7 @@ __global__ void __launch_bounds__(192, 1) softmax_pv_kernel(const __grid_constan
     // Z = O / l (deferred normalisation, line 361)
     mbar_wait_warp(&o_full, 0);
     tc_fence_after();
-    const float inv = l > 0.f ? 1.f / l : 0.f;
+    const float inv = 1.f / l;
     using T = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
 #pragma unroll
     for (int c = 0; c < kDK; c += 32) {
@@ -284,10 +403,9 @@ __global__ void __launch_bounds__(192, 1) softmax_pv_kernel(const __grid_constan
 }
 
 template <bool kBF16, int kDK>
-et_status launch_partial(const CUtensorMap& tm, const CUtensorMap& tv, const PParams& prm, int batch,
-                         unsigned long long* ts_a, cudaStream_t stream) {
-  const size_t smem_a = 1024 + 2 * (kDK / 64) * 16384;
-  const size_t smem_b = 1024 + 2 * 16384 + 2 * (kDK / 64) * 8192;
+et_status launch_partial(const CUtensorMap& tm, const CUtensorMap& ts, const CUtensorMap& tv, const PParams& prm,
+                         int batch, cudaStream_t stream) {
+  const size_t smem_a = QktCfg<kDK>::kSmem, smem_b = PvCfg<kDK>::kSmem;
   static std::once_flag once;
   static cudaError_t err = cudaSuccess;
   std::call_once(once, [&] {
@@ -297,11 +415,9 @@ et_status launch_partial(const CUtensorMap& tm, const CUtensorMap& tv, const PPa
   });
   ET_CUDA(err);
   const int nqb = (prm.S + 127) / 128;
-  PParams pa = prm;
-  pa.ts = ts_a;
-  ET_CUDA(launch_pdl(qkt_kernel<kBF16, kDK>, dim3(nqb, nqb, batch * prm.nh), dim3(128), smem_a, stream, tm, pa));
+  ET_CUDA(launch_pdl(qkt_kernel<kBF16, kDK>, dim3(nqb, batch * prm.nh), dim3(192), smem_a, stream, tm, ts, prm));
   count_launch();
-  ET_CUDA(launch_pdl(softmax_pv_kernel<kBF16, kDK>, dim3(nqb, batch * prm.nh), dim3(192), smem_b, stream, tv, prm));
+  ET_CUDA(launch_pdl(softmax_pv_kernel<kBF16, kDK>, dim3(nqb, batch * prm.nh), dim3(192), smem_b, stream, ts, tv, prm));
   count_launch();
   return ET_OK;
 }
@@ -340,7 +456,6 @@ et_status attention_partial_run(const AttnArgs& a, void* scores, size_t scores_b
   prm.k_off = a.k_off;
   prm.v_off = a.v_off;
   prm.lengths = a.lengths;
-  prm.scores = static_cast<uint16_t*>(scores);
   prm.ld_s = (a.seq_len + 7) / 8 * 8;
   prm.Z = a.Z;
   prm.ld_z = a.ld_z;
@@ -349,12 +464,15 @@ et_status attention_partial_run(const AttnArgs& a, void* scores, size_t scores_b
   prm.box_rows = (int)box_rows;
   prm.vbox_rows = rows < 64 ? (int)rows : 64;
   prm.ts = a.ts;
+  CUtensorMap ts;
+  ET_TRY(make_tmap_3d_ld(&ts, scores, a.dtype, (uint64_t)a.seq_len, (uint64_t)a.seq_len, (uint64_t)a.batch * nh,
+                         (uint64_t)prm.ld_s, 64, 128));
   const bool bf = a.dtype == ET_BF16;
   if (a.d_k == 64)
-    return bf ? launch_partial<true, 64>(tm, tv, prm, a.batch, a.ts, stream)
-              : launch_partial<false, 64>(tm, tv, prm, a.batch, a.ts, stream);
-  return bf ? launch_partial<true, 128>(tm, tv, prm, a.batch, a.ts, stream)
-            : launch_partial<false, 128>(tm, tv, prm, a.batch, a.ts, stream);
+    return bf ? launch_partial<true, 64>(tm, ts, tv, prm, a.batch, stream)
+              : launch_partial<false, 64>(tm, ts, tv, prm, a.batch, stream);
+  return bf ? launch_partial<true, 128>(tm, ts, tv, prm, a.batch, stream)
+            : launch_partial<false, 128>(tm, ts, tv, prm, a.batch, stream);
 }
 
 }  // namespace et

@@ -830,6 +830,25 @@ et_status make_tmap_3d(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t col
   return ET_OK;
 }
 
+// [planes][rows][cols] 16-bit tensor with a row pitch of ld_elems (>= cols), SWIZZLE_128B boxes of
+// box_cols (64) x box_rows; elements outside [cols, rows] read as zero and are dropped on stores
+// (the partial-OTF score matrix, kernels/attention_partial.cu).
+et_status make_tmap_3d_ld(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t cols, uint64_t rows, uint64_t planes,
+                          uint64_t ld_elems, uint32_t box_cols, uint32_t box_rows) {
+  EncodeTiledFn enc = get_encode();
+  if (!enc) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  const uint64_t es = dtype_size(dtype);
+  cuuint64_t dims[3] = {cols, rows, planes};
+  cuuint64_t strides[2] = {ld_elems * es, ld_elems * rows * es};
+  cuuint32_t box[3] = {box_cols, box_rows, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUtensorMapDataType dt = dtype == ET_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  CUresult r = enc(tm, dt, 3, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(ET_ERR_CUDA, "cuTensorMapEncodeTiled (3d, ld) failed (%d)", (int)r);
+  return ET_OK;
+}
+
 // kEpiLN plan: np equal pieces of R tile rows (R even, R <= kLnMaxRows, np <= kLnMaxCluster), the
 // np pieces of a token block forming one cluster; the largest np whose grid fits one wave.
 // OFF unless built with -DET_GEMM_LN_FUSE: measured on C3 (profiles/r01/README.md, v4) the fused

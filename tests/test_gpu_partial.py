@@ -103,7 +103,8 @@ def test_partial_agrees_with_fused_forms(etm, dtype):
     torch.cuda.synchronize()
     ref = oe.attention_core(Q, K, V, H, lens, False, dk=1).reshape(B * S, d)
     assert_close(to64(Zp), ref, **_tol(dtype), what="partial")
-    assert_close(to64(Zp), to64(Zl), **_tol(dtype), what="partial vs long")
+    # both are within _tol of the oracle: they agree within twice that
+    assert_close(to64(Zp), to64(Zl), **{k: 2 * v for k, v in _tol(dtype).items()}, what="partial vs long")
 
 
 def test_partial_head_range_and_bf16_causal(etm):
