@@ -263,6 +263,35 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
                            const float* ln_beta, float ln_eps, void* out, void* workspace, size_t ws_bytes,
                            void* stream);
 
+/* ------------------------------------------------------------------------------------------
+ * Pre-computed linear transformation operator (§3.1 Eq. 4-5, Fig. 3(b)):
+ *   Output = sum_h S_h . X . (W_V,h^T . W_O,h^T) + b'
+ * with the pattern the paper pairs with it (line 107, 317): W_Q / W_K tile-pruned, W_O ROW-pruned
+ * (kept output features `kept`, ascending, n_kept of them), W_V dense.
+ *
+ * et_precompute_vo (offline, once per layer; line 129): Wvo_out device [heads*Dv, d_model] in dtype,
+ *   Dv = round_up(n_kept, 16): row h*Dv + j (j < n_kept) = sum_f W_O[kept[j], h*d_k + f] W_V[h*d_k + f, :]
+ *   (FP32 accumulation of the stored values, rounded once), rows j >= n_kept zero;
+ *   bias_out (optional) device [d_model]: b'[o] = b_O[o] + sum_f W_O[o, f] b_V[f] for kept o, b_O[o]
+ *   otherwise (S_h rows sum to 1, so b_V passes through W_O unchanged; reading C-6).
+ *   Wv, Wo: dense device [d_model, d_model]; bv, bo: [d_model] or NULL.  Pack Wvo_out with
+ *   et_prune_pack(ET_PRUNE_TILE, ratio 0) for et_attention_pre_fwd.
+ * et_attention_pre_fwd: out = SelfAttn(X) (ln_gamma NULL) or LN(X + SelfAttn(X)), X / out [M, d] in
+ *   desc->dtype; wq, wk TILE packed [d, d]; wvo the packed Wvo_out; bq, bk [d]; bias_fold = b'.
+ *   The head sum runs on the tensor core inside the attention kernel (heads of a group accumulate in
+ *   one TMEM accumulator); groups of heads leave partial planes that the LayerNorm step adds.
+ *   Full head range, FP16 / BF16, d_k 64 or 128, seq_len <= 128, d_model <= 4096 (ET_ERR_UNSUPPORTED
+ *   otherwise).  Workspace from et_attention_pre_workspace_size.  Stream-ordered, capturable. */
+et_status et_precompute_vo(const void* Wv, const void* Wo, const void* bv, const void* bo, const int32_t* kept_dev,
+                           int32_t n_kept, int32_t heads, int32_t d_model, et_dtype dtype, void* Wvo_out,
+                           void* bias_out, void* stream);
+et_status et_attention_pre_workspace_size(const et_attn_desc* desc, int32_t n_kept, size_t* bytes);
+et_status et_attention_pre_fwd(const et_attn_desc* desc, const void* X, const et_packed_weight* wq,
+                               const et_packed_weight* wk, const et_packed_weight* wvo, const int32_t* kept_dev,
+                               int32_t n_kept, const void* bq, const void* bk, const void* bias_fold,
+                               const float* ln_gamma, const float* ln_beta, float ln_eps, void* out, void* workspace,
+                               size_t ws_bytes, void* stream);
+
 /* One encoder layer's parameters.  Weights packed; biases in the storage dtype; LN fp32. */
 typedef struct {
   et_packed_weight wq, wk, wv, wo, w1, w2;

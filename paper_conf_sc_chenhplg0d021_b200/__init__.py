@@ -430,6 +430,66 @@ def attention_fwd(X: torch.Tensor, layer: Layer, batch: int, seq_len: int, heads
     return out
 
 
+# ------------------------------------------------------------------- pre-computed operator (Eq. 5)
+_prevo = _sig("et_precompute_vo", ctypes.c_int,
+              [_vp, _vp, _vp, _vp, _vp, _i32, _i32, _i32, ctypes.c_int, _vp, _vp, _vp])
+_pre_ws = _sig("et_attention_pre_workspace_size", ctypes.c_int, [ctypes.POINTER(AttnDescC), _i32, ctypes.POINTER(_sz)])
+_pre = _sig("et_attention_pre_fwd", ctypes.c_int,
+            [ctypes.POINTER(AttnDescC), _vp] + [ctypes.POINTER(PackedWeightC)] * 3 + [_vp, _i32, _vp, _vp, _vp, _vp, _vp,
+                                                                                    _f32, _vp, _vp, _sz, _vp])
+SYMBOLS += ["et_precompute_vo", "et_attention_pre_workspace_size", "et_attention_pre_fwd"]
+
+
+class PreLayer:
+    """Attention block in the pre-computed form (Fig. 3(b)): W_Q / W_K tile
+    pruned, W_O row pruned (kept output features), W_V dense; W_VO = ||_h W_V,h^T W_O,h^T and the folded
+    bias b' computed on the device by et_precompute_vo, W_VO packed as a dense tile weight."""
+
+    def __init__(self, raw: dict, ratio: float, heads: int, dtype="fp16", stream=None):
+        tdt = torch_dtype(dtype)
+        dev = torch.device("cuda")
+        d = raw["wq"].shape[0]
+        self.heads, self.d_model, self.dtype = heads, d, tdt
+        T = {n: torch.as_tensor(raw[n]).to(dev).to(tdt).contiguous() for n in ("wq", "wk", "wv", "wo")}
+        self.wq = prune_pack(T["wq"], "tile", ratio, stream=stream)
+        self.wk = prune_pack(T["wk"], "tile", ratio, stream=stream)
+        self.wo_sel = prune_pack(T["wo"], "row", ratio, stream=stream)    # kept W_O rows = output features
+        self.n_kept = int(self.wo_sel.c.nnz)
+        self.kept = self.wo_sel.kept_index().contiguous()
+        self.Dv = (self.n_kept + 15) // 16 * 16
+        self.dense = {n: torch.as_tensor(raw[n]).to(dev).to(tdt).contiguous() for n in ("bq", "bk", "bv", "bo")}
+        self.dense["ln1_g"] = torch.as_tensor(raw["ln1_g"]).to(dev).to(torch.float32).contiguous()
+        self.dense["ln1_b"] = torch.as_tensor(raw["ln1_b"]).to(dev).to(torch.float32).contiguous()
+        self.wvo_dense = torch.empty(heads * self.Dv, d, dtype=tdt, device=dev)
+        self.bias_fold = torch.empty(d, dtype=tdt, device=dev)
+        _check(_prevo(T["wv"].data_ptr(), T["wo"].data_ptr(), self.dense["bv"].data_ptr(), self.dense["bo"].data_ptr(),
+                      self.kept.data_ptr(), self.n_kept, heads, d, dtype_code(tdt), self.wvo_dense.data_ptr(),
+                      self.bias_fold.data_ptr(), _stream(stream)))
+        self.wvo = prune_pack(self.wvo_dense, "tile", 0.0, stream=stream)
+
+    def workspace_size(self, batch: int, seq_len: int) -> int:
+        d = attn_desc(batch, seq_len, self.heads, self.d_model, self.dtype)
+        nb = _sz()
+        _check(_pre_ws(ctypes.byref(d), self.n_kept, ctypes.byref(nb)))
+        return int(nb.value)
+
+    def __call__(self, X: torch.Tensor, batch: int, seq_len: int, lengths=None, causal=False, ln: bool = True,
+                 ln_eps: float = 1e-12, out=None, workspace=None, stream=None):
+        """et_attention_pre_fwd: LN(X + SelfAttn(X)) (ln=True) or SelfAttn(X)."""
+        d = attn_desc(batch, seq_len, self.heads, self.d_model, X.dtype, lengths, causal)
+        if workspace is None:
+            workspace = torch.empty(self.workspace_size(batch, seq_len), dtype=torch.uint8, device=X.device)
+        if out is None:
+            out = torch.empty(X.shape, dtype=X.dtype, device=X.device)
+        D = self.dense
+        _check(_pre(ctypes.byref(d), X.data_ptr(), ctypes.byref(self.wq.c), ctypes.byref(self.wk.c),
+                    ctypes.byref(self.wvo.c), self.kept.data_ptr(), self.n_kept, D["bq"].data_ptr(), D["bk"].data_ptr(),
+                    self.bias_fold.data_ptr(), D["ln1_g"].data_ptr() if ln else None,
+                    D["ln1_b"].data_ptr() if ln else None, ln_eps, out.data_ptr(), workspace.data_ptr(),
+                    workspace.numel(), _stream(stream)))
+        return out
+
+
 class Encoder:
     """A packed encoder stack bound to a fixed problem shape: owns the C layer array and workspace."""
 

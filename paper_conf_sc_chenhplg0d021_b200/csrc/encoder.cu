@@ -122,7 +122,36 @@ struct BlockWs {
   int32_t* v_width; // [H]
   void* bv_packed;  // [vmax]
   void* bo_folded;  // [d]
+  void* splitk;     // FP32 split-K planes of a K > 768 bias / activation GEMM (d_model > 768), else null
 };
+
+// A GEMM whose epilogue needs whole sums (bias, Q-scale, activation) with K > 768: the tile GEMM
+// holds one 768-column K part of A in TMEM, so it writes FP32 partial planes into `scratch` and
+// splitk_reduce_run adds them and applies the epilogue.  K <= 768 (and partial epilogues): one launch.
+et_status gemm_any(const GemmArgs& g, void* scratch, cudaStream_t st) {
+  if (g.K <= 768 || g.epi == ET_EPI_F32 || g.epi == ET_EPI_PART16 || g.dtype == ET_FP32) return gemm_run(g, st);
+  if (!scratch) return fail(ET_ERR_INTERNAL, "split-K GEMM without scratch");
+  GemmArgs p = g;
+  SplitKSegs sk{};
+  sk.n = g.nseg;
+  int N = 0;
+  for (int s = 0; s < g.nseg; ++s) {
+    sk.col0[s] = g.seg[s].out_col;
+    sk.bias[s] = g.seg[s].bias;
+    sk.scale[s] = g.seg[s].apply_scale ? g.seg[s].scale : 1.0f;
+    N = std::max(N, g.seg[s].out_col + 16 * g.seg[s].tile_rows);
+    p.seg[s].bias = nullptr;
+    p.seg[s].apply_scale = 0;
+  }
+  N = (N + 7) / 8 * 8;
+  p.epi = ET_EPI_F32;
+  p.Y = scratch;
+  p.ldy = N;
+  ET_TRY(gemm_run(p, st));
+  const int act = g.epi == ET_EPI_BIAS_GELU ? 1 : g.epi == ET_EPI_BIAS_RELU ? 2 : 0;
+  return splitk_reduce_run(static_cast<const float*>(scratch), (g.K + 767) / 768, g.M, N, sk, act, g.dtype, g.Y, g.ldy,
+                           st);
+}
 
 int v_cols_of(const et_packed_weight* wv, int d) {   // d: the width W_V produces (inner width)
   return wv->pattern == ET_PRUNE_ROW ? (int)align_up((size_t)std::max(wv->rows_padded, 16), 8) : d;
@@ -133,10 +162,13 @@ int v_cols_of(const et_packed_weight* wv, int d) {   // d: the width W_V produce
 int inner_width(const et_attn_desc* d) { return (d->head_end - d->head_begin) * (d->d_model / d->heads); }
 bool head_parallel(const et_attn_desc* d) { return d->head_begin != 0 || d->head_end != d->heads; }
 
-void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, BlockWs* ws, bool zfull = false) {
+void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, BlockWs* ws, bool zfull = false,
+                 int splitk_cols = 0) {
   const size_t M = (size_t)d->batch * d->seq_len;
   const size_t es = dtype_size(d->dtype);
   const int dq = inner_width(d);
+  const int kp_d = (d->d_model + 767) / 768;
+  kparts_max = std::max(kparts_max, kp_d);   // O-projection partial planes (K = d_model)
   ws->ldq = 2 * dq + vmax;
   ws->qkv = c.take(M * ws->ldq * es);
   ws->z = c.take(M * (zfull ? d->d_model : dq) * es);
@@ -145,6 +177,7 @@ void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, Blo
   ws->v_width = static_cast<int32_t*>(c.take((size_t)d->heads * 4));
   ws->bv_packed = c.take((size_t)vmax * es);
   ws->bo_folded = c.take((size_t)d->d_model * es);
+  ws->splitk = kp_d > 1 ? c.take((size_t)kp_d * M * (std::max(ws->ldq, splitk_cols) + 8) * 4) : nullptr;
 }
 
 // Step 4 fused into the O-projection when possible (kEpiLN: residual in the operand dtype, full head
@@ -208,7 +241,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   g.ldy = ws.ldq;
   g.epi = ET_EPI_BIAS_SCALE;
   g.ts = trace_slot(ET_K_QKV);
-  ET_TRY(gemm_run(g, st));
+  ET_TRY(gemm_any(g, ws.splitk, st));
   // 2. attention core over this call's heads (local indices 0..Hr-1)
   AttnArgs a{};
   a.qkv = ws.qkv;
@@ -313,6 +346,117 @@ et_status et_attn_core_fwd(const et_attn_desc* desc, const void* qkv, int32_t ld
   return attention_run(a, static_cast<cudaStream_t>(stream));
 }
 
+// ---------------------------------------------------------------- pre-computed operator (Eq. 5)
+static int pre_dv(int32_t n_kept) { return (n_kept + 15) / 16 * 16; }
+
+et_status et_precompute_vo(const void* Wv, const void* Wo, const void* bv, const void* bo, const int32_t* kept_dev,
+                           int32_t n_kept, int32_t heads, int32_t d_model, et_dtype dtype, void* Wvo_out,
+                           void* bias_out, void* stream) {
+  if (!Wv || !Wo || (!kept_dev && n_kept > 0) || (!Wvo_out && n_kept > 0))
+    return fail(ET_ERR_INVALID_ARG, "et_precompute_vo: null pointer");
+  if (dtype != ET_FP16 && dtype != ET_BF16) return fail(ET_ERR_UNSUPPORTED, "et_precompute_vo: FP16 / BF16");
+  if (heads <= 0 || d_model <= 0 || d_model % heads) return fail(ET_ERR_INVALID_ARG, "et_precompute_vo: heads / d_model");
+  VoPrep v{Wv, Wo, bv, bo, kept_dev, n_kept, heads, d_model, dtype, Wvo_out, bias_out};
+  return vo_precompute_run(v, static_cast<cudaStream_t>(stream));
+}
+
+static et_status check_pre(const et_attn_desc* desc, const et_packed_weight* wq, const et_packed_weight* wk,
+                           const et_packed_weight* wvo, int32_t n_kept) {
+  ET_TRY(check_desc(desc));
+  if (head_parallel(desc)) return fail(ET_ERR_UNSUPPORTED, "pre-computed operator: full head range only");
+  if (desc->dtype == ET_FP32) return fail(ET_ERR_UNSUPPORTED, "pre-computed operator: FP16 / BF16");
+  if (desc->seq_len > 128) return fail(ET_ERR_UNSUPPORTED, "pre-computed operator: seq_len <= 128");
+  if (n_kept <= 0 || n_kept > desc->d_model) return fail(ET_ERR_INVALID_ARG, "pre-computed operator: n_kept in [1, d_model]");
+  const int dm = desc->d_model;
+  ET_TRY(check_weight(wq, dm, dm, desc->dtype, "W_Q", false));
+  ET_TRY(check_weight(wk, dm, dm, desc->dtype, "W_K", false));
+  ET_TRY(check_weight(wvo, desc->heads * pre_dv(n_kept), dm, desc->dtype, "W_VO", false));
+  return ET_OK;
+}
+
+et_status et_attention_pre_workspace_size(const et_attn_desc* desc, int32_t n_kept, size_t* bytes) {
+  ET_TRY(check_desc(desc));
+  if (!bytes || n_kept <= 0) return fail(ET_ERR_INVALID_ARG, "et_attention_pre_workspace_size");
+  const size_t M = (size_t)desc->batch * desc->seq_len;
+  const int Dv = pre_dv(n_kept), dm = desc->d_model;
+  const int G = attention_pre_groups(desc->batch, desc->heads, Dv);
+  const int kp = (dm + 767) / 768;
+  Carver c{nullptr};
+  c.take(M * (2 * dm + desc->heads * Dv) * dtype_size(desc->dtype));   // Q~ | K | X W_VO
+  c.take((size_t)G * M * dm * 4);                                       // partial planes (sized for FP32)
+  if (kp > 1) c.take((size_t)kp * M * (2 * dm + desc->heads * Dv + 8) * 4);   // split-K planes (d_model > 768)
+  *bytes = c.off + 256;
+  return ET_OK;
+}
+
+et_status et_attention_pre_fwd(const et_attn_desc* desc, const void* X, const et_packed_weight* wq,
+                               const et_packed_weight* wk, const et_packed_weight* wvo, const int32_t* kept_dev,
+                               int32_t n_kept, const void* bq, const void* bk, const void* bias_fold,
+                               const float* ln_gamma, const float* ln_beta, float ln_eps, void* out, void* workspace,
+                               size_t ws_bytes, void* stream) {
+  ET_TRY(check_pre(desc, wq, wk, wvo, n_kept));
+  if (!X || !out || !workspace || !kept_dev) return fail(ET_ERR_INVALID_ARG, "et_attention_pre_fwd: null pointer");
+  size_t need = 0;
+  ET_TRY(et_attention_pre_workspace_size(desc, n_kept, &need));
+  if (ws_bytes < need) return fail(ET_ERR_WORKSPACE, "et_attention_pre_fwd: workspace %zu < %zu", ws_bytes, need);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int dm = desc->d_model, dk = dm / desc->heads, Dv = pre_dv(n_kept);
+  const int M = desc->batch * desc->seq_len;
+  const int G = attention_pre_groups(desc->batch, desc->heads, Dv);
+  Carver c{static_cast<uint8_t*>(workspace)};
+  const int ldq = 2 * dm + desc->heads * Dv;
+  void* qkv = c.take((size_t)M * ldq * dtype_size(desc->dtype));
+  void* planes = c.take((size_t)G * M * dm * 4);
+  void* splitk = dm > 768 ? c.take((size_t)((dm + 767) / 768) * M * (ldq + 8) * 4) : nullptr;
+  // step 1 of Fig. 3(b): X . [W_Q (scaled), W_K, ||_h W_VO,h] in one launch (b_V folded into b')
+  GemmArgs g{};
+  g.X = X;
+  g.M = M;
+  g.K = dm;
+  g.ldx = dm;
+  g.dtype = desc->dtype;
+  g.nseg = 3;
+  g.seg[0] = seg_of(wq, bq, 0);
+  g.seg[0].apply_scale = 1;
+  g.seg[0].scale = 1.0f / std::sqrt((float)dk);
+  g.seg[1] = seg_of(wk, bk, dm);
+  g.seg[2] = seg_of(wvo, nullptr, 2 * dm);
+  g.Y = qkv;
+  g.ldy = ldq;
+  g.epi = ET_EPI_BIAS_SCALE;
+  g.ts = trace_slot(ET_K_QKV);
+  ET_TRY(gemm_any(g, splitk, st));
+  // steps 2-6 and the sum over heads (step 8): G partial planes
+  PreArgs a{};
+  a.qkv = qkv;
+  a.ld_qkv = ldq;
+  a.q_off = 0;
+  a.k_off = dm;
+  a.vo_off = 2 * dm;
+  a.batch = desc->batch;
+  a.seq_len = desc->seq_len;
+  a.heads = desc->heads;
+  a.d_k = dk;
+  a.d = dm;
+  a.Dv = Dv;
+  a.groups = G;
+  a.lengths = desc->lengths_dev;
+  a.kept = kept_dev;
+  a.n_kept = n_kept;
+  a.planes = planes;
+  a.part_dtype = part_dtype_of(desc->dtype);
+  a.causal = desc->causal;
+  a.scale = 1.0f;
+  a.dtype = desc->dtype;
+  a.ts = trace_slot(ET_K_ATTN);
+  ET_TRY(attention_pre_run(a, st));
+  // out = sum of planes + b' (+ X and LN when gamma is given)
+  LnArgs ln{planes, G, M, dm, bias_fold, desc->dtype, ln_gamma ? X : nullptr, desc->dtype, ln_gamma, ln_beta, ln_eps,
+            out, nullptr, nullptr, part_dtype_of(desc->dtype)};
+  ln.ts = trace_slot(ET_K_LN1);
+  return layernorm_run(ln, st);
+}
+
 et_status et_attn_partial_scores_bytes(const et_attn_desc* desc, size_t* bytes) {
   ET_TRY(check_desc(desc));
   if (!bytes) return fail(ET_ERR_INVALID_ARG, "et_attn_partial_scores_bytes: null pointer");
@@ -393,7 +537,7 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   const int M = desc->batch * desc->seq_len;
   // full range: out = part + b_O' (+ X and LN when gamma is given), in dtype;
   // head-parallel: out = FP32 partial (+ b_O' on the rank owning head 0), no residual / LN
-  LnArgs ln{ws.part, 1, M, dm, bo_eff, desc->dtype, ln_gamma ? X : nullptr, hp ? ET_FP32 : desc->dtype, ln_gamma,
+  LnArgs ln{ws.part, wo->kparts, M, dm, bo_eff, desc->dtype, ln_gamma ? X : nullptr, hp ? ET_FP32 : desc->dtype, ln_gamma,
             ln_beta, ln_eps, hp ? nullptr : out, hp ? out : nullptr, nullptr,
             hp ? ET_FP32 : part_dtype_of(desc->dtype)};
   ln.ts = trace_slot(ET_K_LN1);
@@ -415,7 +559,7 @@ et_status et_encoder_workspace_size(const et_attn_desc* desc, int32_t num_layers
   const size_t es = dtype_size(desc->dtype), rs = dtype_size(resid_dtype);
   Carver c{nullptr};
   BlockWs ws;
-  carve_block(c, desc, vmax, kparts, &ws);
+  carve_block(c, desc, vmax, kparts, &ws, false, d_ff);
   c.take(M * d_ff * es);   // U
   c.take(M * dm * es);     // y1 act
   if (resid_dtype != desc->dtype) {
@@ -462,7 +606,7 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
   const int kparts = std::max(1, (d_ff + 767) / 768);
   Carver c{static_cast<uint8_t*>(workspace)};
   BlockWs ws;
-  carve_block(c, desc, vmax, kparts, &ws);
+  carve_block(c, desc, vmax, kparts, &ws, false, d_ff);
   void* U = c.take(M * d_ff * es);
   void* y1a = c.take(M * dm * es);
   const bool split = resid_dtype != desc->dtype;
@@ -487,7 +631,7 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
                                split ? nullptr : &lf));
     // 4. Y1 = LN(X + attn) (unless fused into the O-projection above)
     if (!lf.done) {
-      LnArgs ln1{ws.part, 1, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,
+      LnArgs ln1{ws.part, L.wo.kparts, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,
                  y1a, split ? y1r : nullptr, nullptr, part_dtype_of(desc->dtype)};
       ln1.ts = trace_slot(ET_K_LN1);
       ET_TRY(layernorm_run(ln1, st));
@@ -505,7 +649,7 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     f1.ldy = d_ff;
     f1.epi = act == ET_ACT_GELU_ERF ? ET_EPI_BIAS_GELU : ET_EPI_BIAS_RELU;
     f1.ts = trace_slot(ET_K_FFN1);
-    ET_TRY(gemm_run(f1, st));
+    ET_TRY(gemm_any(f1, ws.splitk, st));
     // 6. U W2'^T -> fp32 split-K partials
     GemmArgs f2{};
     f2.X = U;

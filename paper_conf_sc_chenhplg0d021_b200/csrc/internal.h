@@ -134,6 +134,44 @@ et_status attention32_run(const AttnArgs& a, cudaStream_t stream);
 bool attention128_applies(const AttnArgs& a);
 et_status attention128_run(const AttnArgs& a, cudaStream_t stream);
 int attn_short_max(int d_k);
+// split-K epilogue for K > 768 (kernels/aux.cu): Y = epi(sum of FP32 planes + bias) * scale per segment
+struct SplitKSegs {
+  int n;
+  int col0[3];
+  const void* bias[3];
+  float scale[3];
+};
+et_status splitk_reduce_run(const float* part, int nparts, int M, int N, const SplitKSegs& segs, int act,
+                            et_dtype dtype, void* Y, int ldy, cudaStream_t stream);
+// pre-computed linear transformation (kernels/attention_pre.cu; Eq. 5)
+struct VoPrep {
+  const void* wv;           // [d, d] dense W_V (dtype)
+  const void* wo;           // [d, d] W_O (dtype; rows outside `kept` are treated as pruned)
+  const void* bv;           // [d] or nullptr
+  const void* bo;           // [d] or nullptr
+  const int32_t* kept;      // [n_kept] ascending kept W_O rows
+  int n_kept, heads, d_model;
+  et_dtype dtype;
+  void* wvo_out;            // [heads * Dv, d]
+  void* bias_out;           // [d] or nullptr
+};
+et_status vo_precompute_run(const VoPrep& v, cudaStream_t stream);
+struct PreArgs {
+  const void* qkv;          // [M, ld_qkv]: Q~ at q_off, K at k_off, X W_VO,h at vo_off + h Dv
+  int ld_qkv, q_off, k_off, vo_off;
+  int batch, seq_len, heads, d_k, d, Dv, groups;
+  const int32_t* lengths;
+  const int32_t* kept;
+  int n_kept;
+  void* planes;             // [groups][M][d] in part_dtype
+  et_dtype part_dtype;
+  int causal;
+  float scale;
+  et_dtype dtype;
+  unsigned long long* ts;
+};
+int attention_pre_groups(int batch, int heads, int Dv);
+et_status attention_pre_run(const PreArgs& a, cudaStream_t stream);
 // paper-literal partial OTF (kernels/attention_partial.cu): S = Q K^T materialised in 16 bit,
 // then mask + softmax + x V per row
 size_t attention_partial_scores_bytes(int batch, int seq_len, int heads);

@@ -7,6 +7,7 @@
 #include <cuda_runtime.h>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
+#include <algorithm>
 #include <cstdint>
 
 #include "../internal.h"
@@ -105,6 +106,54 @@ __global__ void vprep_fold_kernel(const uint8_t* __restrict__ wo_values, const i
     stf(bo_folded, dt, i, (float)((bo ? (double)ldf(bo, dt, i) : 0.0) + acc));
 }
 
+
+// Split-K epilogue for K > 768 (one TMEM-resident A part holds 768 columns): Y = epi(sum_p part[p] + b)
+// in the operand dtype.  Segment s covers output columns [col0, col0 + ncols) with its own bias and
+// Q-scale; GELU (reading C-12: the erf form, here evaluated with erff) / ReLU as the GEMM epilogue.
+__global__ void splitk_reduce_kernel(const float* __restrict__ part, int nparts, int M, int N, SplitKSegs segs,
+                                     int act, et_dtype dtype, void* __restrict__ Y, int ldy) {
+  const int n8 = N / 8;
+  const size_t total = (size_t)M * n8;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
+    const int m = (int)(i / n8), c = (int)(i % n8) * 8;
+    float v[8];
+    const float* src = part + (size_t)m * N + c;
+    {
+      const float4 a = *reinterpret_cast<const float4*>(src), b = *reinterpret_cast<const float4*>(src + 4);
+      v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+    }
+    for (int p = 1; p < nparts; ++p) {
+      const float* q = src + (size_t)p * M * N;
+      const float4 a = *reinterpret_cast<const float4*>(q), b = *reinterpret_cast<const float4*>(q + 4);
+      v[0] += a.x; v[1] += a.y; v[2] += a.z; v[3] += a.w; v[4] += b.x; v[5] += b.y; v[6] += b.z; v[7] += b.w;
+    }
+    int s = 0;
+    while (s + 1 < segs.n && c >= segs.col0[s + 1]) ++s;
+    const void* bias = segs.bias[s];
+    const float scale = segs.scale[s];
+    for (int u = 0; u < 8; ++u) {
+      float x = v[u];
+      if (bias) x += dtype == ET_BF16 ? __bfloat162float(static_cast<const __nv_bfloat16*>(bias)[c - segs.col0[s] + u])
+                                      : __half2float(static_cast<const __half*>(bias)[c - segs.col0[s] + u]);
+      if (act == 1) x = 0.5f * x * (1.0f + erff(x * 0.70710678118654752f));
+      else if (act == 2) x = fmaxf(x, 0.0f);
+      v[u] = x * scale;
+    }
+    uint4 o;
+    uint32_t* ow = reinterpret_cast<uint32_t*>(&o);
+    for (int u = 0; u < 4; ++u) {
+      if (dtype == ET_BF16) {
+        __nv_bfloat162 h = __floats2bfloat162_rn(v[2 * u], v[2 * u + 1]);
+        ow[u] = *reinterpret_cast<uint32_t*>(&h);
+      } else {
+        __half2 h = __floats2half2_rn(v[2 * u], v[2 * u + 1]);
+        ow[u] = *reinterpret_cast<uint32_t*>(&h);
+      }
+    }
+    *reinterpret_cast<uint4*>(static_cast<uint16_t*>(Y) + (size_t)m * ldy + c) = o;
+  }
+}
+
 }  // namespace
 
 et_status cast_run(const void* src, et_dtype sdt, void* dst, et_dtype ddt, size_t n, cudaStream_t stream) {
@@ -138,6 +187,17 @@ et_status vprep_run(const VPrep& v, cudaStream_t stream) {
                                                          v.bo_folded);
   count_launch();
   ET_CUDA(cudaGetLastError());
+  return ET_OK;
+}
+
+et_status splitk_reduce_run(const float* part, int nparts, int M, int N, const SplitKSegs& segs, int act,
+                            et_dtype dtype, void* Y, int ldy, cudaStream_t stream) {
+  if (N % 8 || (ldy * 2) % 16 || !aligned16(Y)) return fail(ET_ERR_INVALID_ARG, "split-K reduce: 16-byte rows required");
+  const size_t total = (size_t)M * (N / 8);
+  const int grid = (int)std::min<size_t>((total + 255) / 256, 148 * 8);
+  splitk_reduce_kernel<<<grid, 256, 0, stream>>>(part, nparts, M, N, segs, act, dtype, Y, ldy);
+  ET_CUDA(cudaGetLastError());
+  count_launch();
   return ET_OK;
 }
 

@@ -195,7 +195,11 @@ __device__ __forceinline__ void layernorm_row8(const LnArgs& a) {
   const void* bias_p = has_bias ? a.bias : a.part;   // dummy addresses for absent operands: the loads
   const void* res_p = has_res ? a.resid : a.part;    // stay unconditional, the values are discarded
   float v[NCH][8];
-  float part[NP][NCH][8], bias[NCH][8], res[NCH][8];
+  // up to 16 (chunk, partial) pairs: every partial of the row in registers before any arithmetic
+  // (loads in flight); wider rows or more partials (d_model 2048, d_ff 4096: Fig. 9) fold the
+  // partials chunk by chunk (register budget)
+  constexpr int NPR = NCH * NP <= 16 ? NP : 1;
+  float part[NPR][NCH][8], bias[NCH][8], res[NCH][8];
   bool ok[NCH];
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
@@ -204,8 +208,14 @@ __device__ __forceinline__ void layernorm_row8(const LnArgs& a) {
 #pragma unroll
     for (int q = 0; q < NP; ++q) {
       const size_t off = (size_t)q * a.M * a.N + row + col;
-      if constexpr (P16) ld8<DT>(a.part, off, part[q][c]);
-      else ld8<ET_FP32>(a.part, off, part[q][c]);
+      float t[8];
+      if constexpr (P16) ld8<DT>(a.part, off, t);
+      else ld8<ET_FP32>(a.part, off, t);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        if constexpr (NPR == NP) part[q][c][e] = t[e];
+        else part[0][c][e] = q == 0 ? t[e] : part[0][c][e] + t[e];
+      }
     }
     ld8<DT>(bias_p, has_bias ? col : 0, bias[c]);
     ld8<RT>(res_p, has_res ? row + col : 0, res[c]);
@@ -217,7 +227,7 @@ __device__ __forceinline__ void layernorm_row8(const LnArgs& a) {
     for (int e = 0; e < 8; ++e) {
       float x = part[0][c][e];
 #pragma unroll
-      for (int q = 1; q < NP; ++q) x += part[q][c][e];
+      for (int q = 1; q < NPR; ++q) x += part[q][c][e];
       // absent operands / out-of-range lanes masked by a bit AND (see layernorm_row)
       x += __uint_as_float(__float_as_uint(bias[c][e]) & (has_bias ? 0xffffffffu : 0u));
       x += __uint_as_float(__float_as_uint(res[c][e]) & (has_res ? 0xffffffffu : 0u));
@@ -287,7 +297,18 @@ et_status launch_np(const LnArgs& a, cudaStream_t stream) {
     case 2: e = launch_pdl(layernorm_kernel<NCH, 2, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
     case 3: e = launch_pdl(layernorm_kernel<NCH, 3, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
     case 4: e = launch_pdl(layernorm_kernel<NCH, 4, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
-    default: return fail(ET_ERR_UNSUPPORTED, "LayerNorm: up to 4 partial inputs (got %d)", a.nparts);
+    default:
+      if constexpr (NCH < 0) {   // 8-wide form only: more K parts (K > 3072)
+        switch (a.nparts) {
+          case 5: e = launch_pdl(layernorm_kernel<NCH, 5, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
+          case 6: e = launch_pdl(layernorm_kernel<NCH, 6, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
+          case 7: e = launch_pdl(layernorm_kernel<NCH, 7, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
+          case 8: e = launch_pdl(layernorm_kernel<NCH, 8, DT, RT, P16>, dim3(blocks), dim3(threads), 0, stream, a); break;
+          default: return fail(ET_ERR_UNSUPPORTED, "LayerNorm: up to 8 partial inputs (got %d)", a.nparts);
+        }
+        break;
+      }
+      return fail(ET_ERR_UNSUPPORTED, "LayerNorm: up to 4 partial inputs with N %% 8 != 0 (got %d)", a.nparts);
   }
   ET_CUDA(e);
   count_launch();
@@ -316,17 +337,19 @@ et_status launch_dt(const LnArgs& a, cudaStream_t stream) {
 }  // namespace
 
 et_status layernorm_run(const LnArgs& a, cudaStream_t stream) {
-  if (a.N % 4 || a.N > 128 * 8)
-    return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 4 and <= 1024 (got %d)", a.N);
+  if (a.N % 4 || a.N > 256 * 8 || (a.N > 128 * 8 && a.N % 8))
+    return fail(ET_ERR_UNSUPPORTED, "LayerNorm: N must be a multiple of 4 and <= 1024, or of 8 and <= 2048 (got %d)", a.N);
   if (a.M <= 0) return ET_OK;
-  // 8-wide form (16-byte accesses) for up to 4 partial inputs (more partials: the 4-wide form,
-  // whose smaller per-lane register footprint keeps more rows in flight)
-  if (a.N % 8 == 0 && a.nparts <= 4) {
+  // 8-wide form (16-byte accesses) whenever N % 8 == 0 (up to 8 partial inputs); the 4-wide form
+  // for N % 8 == 4
+  if (a.N % 8 == 0 && a.nparts <= 8) {
     switch ((a.N + 255) / 256) {
       case 1: return launch_dt<-1>(a, stream);
       case 2: return launch_dt<-2>(a, stream);
       case 3: return launch_dt<-3>(a, stream);
-      default: return launch_dt<-4>(a, stream);
+      case 4: return launch_dt<-4>(a, stream);
+      case 5: case 6: return launch_dt<-6>(a, stream);
+      default: return launch_dt<-8>(a, stream);
     }
   }
   switch ((a.N + 127) / 128) {

@@ -1,10 +1,9 @@
 #!/bin/bash
-# One gpurun call: GPU tests, smoke, default bench, then the ncu launch list + full captures.
+# full GPU test suite, then optional sweeps (args: sweep names for tools/sweeps.py)
 mkdir -p gpurun_out
-nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/smi.txt 2>&1
-timeout 900 python -m pytest tests -m gpu -q -x 2>&1 | tail -30 > gpurun_out/pytest_gpu.log
-timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
-timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err
-timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
-if [ "$1" == "prof" ]; then timeout 1500 bash tools/profile_round.sh > gpurun_out/prof.log 2>&1; fi
-ls -la gpurun_out
+timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -30 > gpurun_out/gpu_tests.log
+tail -5 gpurun_out/gpu_tests.log
+if [ -n "$1" ]; then
+  timeout 900 python tools/sweeps.py "$@" > gpurun_out/sweeps.jsonl 2> gpurun_out/sweeps.err
+  cat gpurun_out/sweeps.jsonl; tail -5 gpurun_out/sweeps.err
+fi

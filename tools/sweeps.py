@@ -3,7 +3,8 @@
       tokens for d x d (d = 768, 1024) and the BERT FFN shapes, tile ratio 0 ... 0.95;
   M3  sequence-length crossover (Fig. 8 / line 244 analogue): short vs long attention form vs the
       paper-literal partial OTF at fixed total tokens, BERT-base heads (H = 12, d_k = 64);
-  M3b the same at batch 1 (Fig. 8's setting), BERT-base and Transformer heads.
+  M3b the same at batch 1 (Fig. 8's setting), BERT-base and Transformer heads;
+  M4  pre-computed linear transformation vs the standard attention block (Fig. 9 / line 248-250).
 Timing: CUDA events around 50 back-to-back launches after 5 warm-ups (operands L2-resident when they
 fit: a kernel-level diagnostic, not the bench metric).  Dense torch.matmul at the same shape is
 printed as context only (it is never a backend)."""
@@ -147,8 +148,39 @@ def m3b():
             _m3_row("M3b", S, 1, H, 64)
 
 
+def m4(batch=32):
+    """Fig. 9 analogue (§5.2.3): the attention block (steps 1-8
+    and the residual + LayerNorm) with vs without the pre-computed linear transformation, S = 128,
+    d in {768, 1024, 2048}, heads with d_k in {64, 128}.  The paper prunes 50 % without and 80 % with
+    the pre-computed operator (its accuracy budget); the 80 %-vs-80 % pair is printed too.  Without:
+    W_Q/W_K/W_O tile, W_V row (attention-aware); with: W_Q/W_K tile, W_O row, W_V dense."""
+    from et_synth import CONFIGS, make_layer, make_x
+    S = 128
+    for d in (768, 1024, 2048):
+        for H in (d // 128, d // 64):
+            cfg = CONFIGS["C2"].with_(d_model=d, heads=H, d_ff=4 * d, seq_len=S, batch=batch, layers=1)
+            raw = make_layer(cfg, 0)
+            X = torch.tensor(make_x(cfg).reshape(batch * S, d), dtype=torch.float16, device="cuda")
+            row = {"sweep": "M4", "d": d, "H": H, "d_k": d // H, "S": S, "B": batch}
+            for ratio in (0.5, 0.8):
+                lay = et.pack_layer(raw, "attention-aware", ratio, H, "fp16")
+                ws = torch.empty(et.attention_workspace_size(lay, batch, S, H, d, torch.float16), dtype=torch.uint8,
+                                 device="cuda")
+                out = torch.empty_like(X)
+                row[f"std_{int(ratio * 100)}_us"] = round(timed(
+                    lambda: et.attention_fwd(X, lay, batch, S, H, out=out, workspace=ws)), 2)
+            pre = et.PreLayer(raw, 0.8, H, "fp16")
+            wsp = torch.empty(pre.workspace_size(batch, S), dtype=torch.uint8, device="cuda")
+            outp = torch.empty_like(X)
+            row["pre_80_us"] = round(timed(lambda: pre(X, batch, S, out=outp, workspace=wsp)), 2)
+            row["pre_Dv"] = pre.Dv
+            row["speedup_pre80_vs_std50"] = round(row["std_50_us"] / row["pre_80_us"], 3)
+            row["speedup_pre80_vs_std80"] = round(row["std_80_us"] / row["pre_80_us"], 3)
+            print(json.dumps(row), flush=True)
+
+
 if __name__ == "__main__":
-    which = sys.argv[1:] or ["m2", "m2b", "m3", "m3b"]
+    which = sys.argv[1:] or ["m2", "m2b", "m3", "m3b", "m4"]
     if "m2" in which:
         m2()
     if "m2b" in which:
@@ -157,3 +189,5 @@ if __name__ == "__main__":
         m3()
     if "m3b" in which:
         m3b()
+    if "m4" in which:
+        m4()
