@@ -259,6 +259,23 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   constexpr int a_rot = 0;
 #endif
   auto a_chunk = [&](int sq) { return sq + a_rot < nk ? sq + a_rot : sq + a_rot - nk; };
+  // Ring positions (position s uses slot s % kSlots and recycles position s - kSlots): the A chunks,
+  // then the tile chunks.  -DET_GEMM_T0_EARLY moves the first tile chunk ahead of the A chunks that
+  // do not fit the ring (into A chunk 0's slot) so that it lands with the A block: measured slower on
+  // C3 (every GEMM +0.5-0.7 us, 40.4k -> 38.9k seq/s; the delayed A chunks are the critical path).
+#ifdef ET_GEMM_T0_EARLY
+  const int t0_early = (nk > kSlots && nchunks > 0) ? 1 : 0;
+#else
+  constexpr int t0_early = 0;
+#endif
+  auto pos_a = [&](int sq) { return sq + (t0_early && sq >= kSlots ? 1 : 0); };
+  auto pos_t = [&](int c) { return t0_early && c == 0 ? kSlots : nk + c; };
+  // position -> load: >= 0 A chunk (load order index), < 0 tile chunk -(c + 1)
+  auto at_pos = [&](int s) {
+    if (t0_early && s == kSlots) return -1;
+    const int sa_ = s - (t0_early && s > kSlots ? 1 : 0);
+    return s < nk + t0_early ? sa_ : -(s - nk + 1);
+  };
   if (threadIdx.x == 0) ET_TL(0);
   ET_TL_RESET();
 #ifdef ET_TIMELINE
@@ -313,7 +330,7 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
     for (int sq = warp >> 2; sq < nk; sq += kFillSets) {   // load sequence position sq holds chunk j
       const int j = a_chunk(sq);
       mbar_wait_warp(&bar.xfull[sq], 0);
-      const uint8_t* rowp = ring + (sq % kSlots) * kSlotBytes + rr * 128;
+      const uint8_t* rowp = ring + (pos_a(sq) % kSlots) * kSlotBytes + rr * 128;
       uint32_t v[32];
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
@@ -350,10 +367,11 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
         const int slot = s % kSlots;
         const int prev = s - kSlots;
         if (prev >= 0) {
-          if (prev < nk) {
-            mbar_wait(&bar.xfree[prev], 0);
+          const int lp = at_pos(prev);
+          if (lp >= 0) {
+            mbar_wait(&bar.xfree[lp], 0);
           } else {
-            const int end_rel = (prev - nk + 1) * kChunkTiles;
+            const int end_rel = (-lp) * kChunkTiles;   // tile chunk -lp - 1 ends here
             while (tl + 1 < nrows && bar.rptr[tl + 1] < end_rel) ++tl;
             // pair slots 0 .. tl / 2 (rows 0 .. tl) observed complete
             while (pdone <= (tl >> 1)) {
@@ -363,11 +381,12 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
           }
         }
         uint8_t* dst = ring + slot * kSlotBytes;
-        if (s < nk) {
-          mbar_expect_tx(&bar.xfull[s], p.box_rows * 128);
-          tma_load_2d(dst, &tmap_x, &bar.xfull[s], kx0 + a_chunk(s) * 64, m0);
+        const int ls = at_pos(s);
+        if (ls >= 0) {
+          mbar_expect_tx(&bar.xfull[ls], p.box_rows * 128);
+          tma_load_2d(dst, &tmap_x, &bar.xfull[ls], kx0 + a_chunk(ls) * 64, m0);
         } else {
-          const int c = s - nk;
+          const int c = -ls - 1;
           const bool inB = c >= nchA;
           const SegDev& sx = inB ? sb : sa;
           const int cc = inB ? c - nchA : c, pbx = inB ? pbB : pbA, pex = inB ? peB : peA;
@@ -416,7 +435,7 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
           cur_chunk = c;
           tc_fence_after();
         }
-        const int slot = (nk + c) % kSlots;
+        const int slot = pos_t(c) % kSlots;
         const int coff = two ? bar.tcoff[slot] : (pbA + c * kChunkTiles) & 3;
         n = qe - qb;
         mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
