@@ -76,9 +76,11 @@ def build_diag(verbose: bool = False) -> str:
 
 
 def build(verbose: bool = False, force: bool = False, debug: bool = False, variant: str | None = None,
-          defines: tuple[str, ...] = ()) -> str:
+          defines: tuple[str, ...] = (), only: str | None = None) -> str:
     """Compile every .cu and link libet.so (debug=True: -DET_WATCHDOG build into build/et_dbg/libet_dbg.so;
-    variant=NAME: an experiment build with extra -D defines into build/et_var_NAME/libet.so)."""
+    variant=NAME: an experiment build with extra -D defines into build/et_var_NAME/libet.so; only=SUBSTR:
+    compile just the sources whose name contains SUBSTR with those defines and link the main build's
+    objects for the rest)."""
     nvcc = _nvcc()
     if variant:
         bdir = BUILD + "_var_" + variant
@@ -93,6 +95,9 @@ def build(verbose: bool = False, force: bool = False, debug: bool = False, varia
     objs = []
     for src in sources():
         rel = os.path.relpath(src, CSRC).replace(os.sep, "_")
+        if variant and only and only not in rel:
+            objs.append(os.path.join(BUILD, rel + ".o"))   # the main build's object
+            continue
         obj = os.path.join(bdir, rel + ".o")
         objs.append(obj)
         if force or not os.path.exists(obj) or os.path.getmtime(obj) < max(os.path.getmtime(src), hdr_mtime):
@@ -129,6 +134,8 @@ def build(verbose: bool = False, force: bool = False, debug: bool = False, varia
 if __name__ == "__main__":
     var = sys.argv[sys.argv.index("--variant") + 1] if "--variant" in sys.argv else None
     defs = tuple(a[2:] for a in sys.argv if a.startswith("-D"))
-    print(build(verbose=True, force="--force" in sys.argv, debug="--debug" in sys.argv, variant=var, defines=defs))
+    only = sys.argv[sys.argv.index("--only") + 1] if "--only" in sys.argv else None
+    print(build(verbose=True, force="--force" in sys.argv, debug="--debug" in sys.argv, variant=var, defines=defs,
+                only=only))
     if "--diag" in sys.argv:
         print(build_diag(verbose=True))

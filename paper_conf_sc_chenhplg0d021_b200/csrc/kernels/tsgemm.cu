@@ -210,6 +210,14 @@ __device__ __forceinline__ void gelu_erf2(float& x0, float& x1) {
 // epilogues that write raw accumulators (no bias) as split-K partial planes [kparts][M][ldy]
 constexpr bool is_partial(int e) { return e == ET_EPI_F32 || e == ET_EPI_PART16; }
 
+// Accumulator hand-off waits (MMA warp <- epilogue drain, epilogue <- MMA commit).  -DET_GEMM_SPIN:
+// spin without the suspend-time hint (a parked waiter's wake-up sits on the round's critical path).
+#ifdef ET_GEMM_SPIN
+#define GEMM_HANDOFF_WAIT(b, ph) mbar_wait_fast_warp((b), (ph))
+#else
+#define GEMM_HANDOFF_WAIT(b, ph) mbar_wait_warp((b), (ph))
+#endif
+
 template <int kEpi, bool kBF16>
 __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
                                                              const __grid_constant__ CUtensorMap tmap_y,
@@ -448,7 +456,7 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
       };
       if (qb < q1) prep();
       if (k > 0) {   // the epilogue group must have read this accumulator's previous row
-        mbar_wait_warp(&bar.acc_empty[acc], (k - 1) & 1);
+        GEMM_HANDOFF_WAIT(&bar.acc_empty[acc], (k - 1) & 1);
         tc_fence_after();
       }
       if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k);
@@ -513,7 +521,7 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
         for (int ch = 0; ch < 4; ++ch) res4[ch] = __ldg(rp4 + ch);
       }
       (void)k;
-      mbar_wait_warp(&bar.slot_full[jp], 0);   // single-use: both rows' MMAs complete
+      GEMM_HANDOFF_WAIT(&bar.slot_full[jp], 0);   // single-use: both rows' MMAs complete
       if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it);
       tc_fence_after();
       if (quarter == 0 && lane == 0)   // the pair's MMAs are complete: their tiles are free
@@ -606,7 +614,12 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
       // output columns: segments of a two-part piece are output-contiguous (checked on the host)
       const int col0 = t0 < rowsA ? sa.out_col + (pc.i0 + t0) * 16 : sb.out_col + (t0 - rowsA) * 16;
       const int row0 = m0 + quarter * 32;
-      if (na == 2) {
+#ifdef ET_GEMM_DIRECT_ST
+      constexpr bool kDirect = !kLN;
+#else
+      constexpr bool kDirect = false;
+#endif
+      if (na == 2 && !kDirect) {
         if (lane == 0) bulk_wait_group_read<0>();   // the previous store finished reading the staging tile
         __syncwarp();
         if constexpr (kEpi == ET_EPI_F32) {
@@ -633,22 +646,27 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
           bulk_commit_group();
         }
       } else {
-        // a lone last row of the piece: direct stores of its 16 columns only, so nothing is written
-        // into the neighbouring piece's or segment's columns
+        // direct stores (-DET_GEMM_DIRECT_ST: every pair; otherwise a lone last row of the piece, so
+        // nothing is written into the neighbouring piece's or segment's columns): 16 columns per row
         const int row = row0 + lane;
         if (row < p.M) {
-          if constexpr (kEpi == ET_EPI_F32) {
-            float* y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row * p.ldy + col0;
 #pragma unroll
-            for (int c = 0; c < 16; c += 4)
-              *reinterpret_cast<float4*>(y + c) = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
-          } else {
-            uint16_t* y = static_cast<uint16_t*>(p.Y) + (kEpi == ET_EPI_PART16 ? (size_t)z * p.part_stride : 0) +
-                          (size_t)row * p.ldy + col0;
-            *reinterpret_cast<uint4*>(y) = make_uint4(pack2<kBF16>(v[0], v[1]), pack2<kBF16>(v[2], v[3]),
-                                                      pack2<kBF16>(v[4], v[5]), pack2<kBF16>(v[6], v[7]));
-            *reinterpret_cast<uint4*>(y + 8) = make_uint4(pack2<kBF16>(v[8], v[9]), pack2<kBF16>(v[10], v[11]),
-                                                          pack2<kBF16>(v[12], v[13]), pack2<kBF16>(v[14], v[15]));
+          for (int a = 0; a < 2; ++a) {
+            if (a >= na) break;
+            const float* va = v + 16 * a;
+            if constexpr (kEpi == ET_EPI_F32) {
+              float* y = static_cast<float*>(p.Y) + (size_t)z * p.part_stride + (size_t)row * p.ldy + col0 + 16 * a;
+#pragma unroll
+              for (int c = 0; c < 16; c += 4)
+                *reinterpret_cast<float4*>(y + c) = make_float4(va[c], va[c + 1], va[c + 2], va[c + 3]);
+            } else {
+              uint16_t* y = static_cast<uint16_t*>(p.Y) + (kEpi == ET_EPI_PART16 ? (size_t)z * p.part_stride : 0) +
+                            (size_t)row * p.ldy + col0 + 16 * a;
+              *reinterpret_cast<uint4*>(y) = make_uint4(pack2<kBF16>(va[0], va[1]), pack2<kBF16>(va[2], va[3]),
+                                                        pack2<kBF16>(va[4], va[5]), pack2<kBF16>(va[6], va[7]));
+              *reinterpret_cast<uint4*>(y + 8) = make_uint4(pack2<kBF16>(va[8], va[9]), pack2<kBF16>(va[10], va[11]),
+                                                            pack2<kBF16>(va[12], va[13]), pack2<kBF16>(va[14], va[15]));
+            }
           }
         }
       }
