@@ -190,7 +190,8 @@ template <int kEpi> struct Smem {
 // transformed exactly; the clamp moves to |x| = 4 sqrt 2, where |nu e| < 5e-8): |GELU error| <= 1.6e-6
 // (float32 emulation of this code against the float64 erf form), below FP16/BF16 output resolution
 // for |GELU| > 4e-3.  Degree 4 instead of 5: one packed FMA less per pair — FFN1 15.3 -> 14.7 us per
-// C3 layer (A/B on one box), the epilogue being issue-bound.  Two elements at a time: one FMNMX per
+// C3 layer (A/B on one box), the epilogue being issue-bound.  (ex2.approx.f16x2 on the pair - half
+// the MUFU ops, two more conversions - measured slower: FFN1 14.4 -> 15.1 us, profiles/r02.)  Two elements at a time: one FMNMX per
 // element for nu (the -|x| operand modifier), 6 packed FP32x2 FMAs and two MUFU.EX2 per pair.
 __device__ __forceinline__ void gelu_erf2(float& x0, float& x1) {
   const uint64_t nu = f2pk(fmaxf(-fabsf(x0), -5.65685424949238f), fmaxf(-fabsf(x1), -5.65685424949238f));
@@ -256,8 +257,6 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   const int nrounds = (nrows + kAcc - 1) / kAcc;   // row t: accumulator t % 8, round t / 8
   const int npairs_all = (nrows + 1) / 2;          // pair slots
 
-  if (nchunks > kMaxBChunks || nrows > kMaxRows || (!is_partial(kEpi) && nrows > kMaxBiasRows))
-    __trap();   // host sizes pieces so this cannot happen
   // A chunks are loaded in K order (the first round's MMAs follow the fill chunk by chunk).
   // ET_GEMM_A_ROT: rotate the order per piece instead (CTAs of one token block start a quarter of
   // the block apart) — measured no faster: the L2 serves the sharing CTAs well (profiles/r01).
@@ -267,23 +266,32 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   constexpr int a_rot = 0;
 #endif
   auto a_chunk = [&](int sq) { return sq + a_rot < nk ? sq + a_rot : sq + a_rot - nk; };
-  // Ring positions (position s uses slot s % kSlots and recycles position s - kSlots): the A chunks,
-  // then the tile chunks.  -DET_GEMM_T0_EARLY moves the first tile chunk ahead of the A chunks that
-  // do not fit the ring (into A chunk 0's slot) so that it lands with the A block: measured slower on
-  // C3 (every GEMM +0.5-0.7 us, 40.4k -> 38.9k seq/s; the delayed A chunks are the critical path).
-#ifdef ET_GEMM_T0_EARLY
-  const int t0_early = (nk > kSlots && nchunks > 0) ? 1 : 0;
-#else
-  constexpr int t0_early = 0;
-#endif
-  auto pos_a = [&](int sq) { return sq + (t0_early && sq >= kSlots ? 1 : 0); };
-  auto pos_t = [&](int c) { return t0_early && c == 0 ? kSlots : nk + c; };
+  // Ring positions: position s uses slot s % kSlots and recycles position s - kSlots; the A chunks
+  // come first (positions 0 .. nk - 1), then the tile chunks.  (-DET_GEMM_T0_EARLY, the first tile
+  // chunk moved ahead of the A chunks that do not fit the ring, measured slower: every GEMM
+  // +0.5-0.7 us on C3, profiles/r02/ab_gemm_t0_early.txt; removed.)
+  auto pos_t = [&](int c) { return nk + c; };
   // position -> load: >= 0 A chunk (load order index), < 0 tile chunk -(c + 1)
-  auto at_pos = [&](int s) {
-    if (t0_early && s == kSlots) return -1;
-    const int sa_ = s - (t0_early && s > kSlots ? 1 : 0);
-    return s < nk + t0_early ? sa_ : -(s - nk + 1);
-  };
+  auto at_pos = [&](int s) { return s < nk ? s : -(s - nk + 1); };
+  // The producer issues the A loads that need no slot recycling (positions < kSlots) before the
+  // block-wide setup: they depend only on the launch geometry, while the setup waits on global loads
+  // of the weight's row pointers (measured ~1-1.5k cycles at kernel start, profiles/r02).
+  const int n_early = min(nk, kSlots);
+  if (warp == kWarpP && lane == 0) {
+    for (int i = 0; i < kMaxKChunks; ++i) {
+      mbar_init(&bar.xfull[i], 1);
+      mbar_init(&bar.xfree[i], 4);
+    }
+    mbar_init(&bar.a_all, 4 * nk);
+    fence_mbar_init();
+    tma_prefetch_desc(&tmap_x);
+    pdl_wait();
+    if (p.ts != nullptr) atomicMin(p.ts, globaltimer_ns());   // trace: this CTA's work starts
+    for (int s = 0; s < n_early; ++s) {
+      mbar_expect_tx(&bar.xfull[s], p.box_rows * 128);
+      tma_load_2d(ring + s * kSlotBytes, &tmap_x, &bar.xfull[s], z * p.Kp + a_chunk(s) * 64, m0);
+    }
+  }
   if (threadIdx.x == 0) ET_TL(0);
   ET_TL_RESET();
 #ifdef ET_TIMELINE
@@ -296,11 +304,8 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   }
 #endif
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kMaxKChunks; ++i) {
-      mbar_init(&bar.xfull[i], 1);
-      mbar_init(&bar.xfree[i], 4);
-    }
-    mbar_init(&bar.a_all, 4 * nk);
+    if (nchunks > kMaxBChunks || nrows > kMaxRows || (!is_partial(kEpi) && nrows > kMaxBiasRows))
+      __trap();   // host sizes pieces so this cannot happen
     for (int i = 0; i < kAcc; ++i) mbar_init(&bar.acc_empty[i], 4);
     for (int j = 0; j < npairs_all; ++j) mbar_init(&bar.slot_full[j], min(2, nrows - 2 * j));   // one commit per row
     for (int i = 0; i < nchunks; ++i) mbar_init(&bar.bfull[i], 1);
@@ -338,7 +343,7 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
     for (int sq = warp >> 2; sq < nk; sq += kFillSets) {   // load sequence position sq holds chunk j
       const int j = a_chunk(sq);
       mbar_wait_warp(&bar.xfull[sq], 0);
-      const uint8_t* rowp = ring + (pos_a(sq) % kSlots) * kSlotBytes + rr * 128;
+      const uint8_t* rowp = ring + (sq % kSlots) * kSlotBytes + rr * 128;
       uint32_t v[32];
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
@@ -364,14 +369,11 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
     // rows being 8k + 2g + {0, 1}).  A row spans at most 3 tile chunks < kSlots, so the producer
     // never waits for a row that itself needs the chunk being loaded.
     if (lane == 0) {
-      tma_prefetch_desc(&tmap_x);
-      pdl_wait();
-      if (p.ts != nullptr) atomicMin(p.ts, globaltimer_ns());   // trace: this CTA's work starts
       const int kx0 = z * p.Kp;
       int tl = 0;   // last local row that starts before the end of the tile chunk being recycled
       int pdone = 0;   // pair slots [0, pdone) known complete
       const int nseq = nk + nchunks;
-      for (int s = 0; s < nseq; ++s) {
+      for (int s = n_early; s < nseq; ++s) {   // positions < n_early: issued before the setup
         const int slot = s % kSlots;
         const int prev = s - kSlots;
         if (prev >= 0) {
