@@ -56,6 +56,7 @@ def _case(key, **kw):
     ("C2", {}),
     ("C3", {"layers": 2, "batch": 4}),
     ("C3", {"layers": 2, "batch": 3, "dtype": "bf16"}),
+    ("C3", {"layers": 2, "batch": 3, "seq_len": 80}),   # M = 240: a ragged last token block
     ("C4", {"layers": 1, "batch": 2}),
     ("C5", {"layers": 1, "batch": 1}),
 ])
