@@ -649,7 +649,6 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     f1.ldy = d_ff;
     f1.epi = act == ET_ACT_GELU_ERF ? ET_EPI_BIAS_GELU : ET_EPI_BIAS_RELU;
     f1.ts = trace_slot(ET_K_FFN1);
-    ET_TRY(gemm_any(f1, ws.splitk, st));
     // 6. U W2'^T -> fp32 split-K partials
     GemmArgs f2{};
     f2.X = U;
@@ -663,7 +662,17 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     f2.ldy = dm;
     f2.epi = part_epi_of(desc->dtype);
     f2.ts = trace_slot(ET_K_FFN2);
-    ET_TRY(gemm_run(f2, st));
+#ifdef ET_NO_FFN_FUSE
+    const bool ffn_fused = false;   // A/B switch (compile time)
+#else
+    const bool ffn_fused = gemm_ffn_applies(f1, f2);
+#endif
+    if (ffn_fused) {   // one launch: FFN1 piece c, then FFN2 K part c, per CTA
+      ET_TRY(gemm_ffn_run(f1, f2, st));
+    } else {
+      ET_TRY(gemm_any(f1, ws.splitk, st));
+      ET_TRY(gemm_run(f2, st));
+    }
     // 7. Y2 = LN(Y1 + F + b2)
     LnArgs ln2{ws.part, L.w2.kparts, (int)M, dm, L.b2, desc->dtype, y1r, resid_dtype, L.ln2_g, L.ln2_b, ln_eps,
                split ? next_act : nullptr, next_res, nullptr, part_dtype_of(desc->dtype)};

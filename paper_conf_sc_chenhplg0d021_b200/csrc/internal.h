@@ -86,6 +86,9 @@ constexpr int kEpiLN = 16;
 // true if gemm_run can run `a` with kEpiLN (shape / dtype / piece constraints)
 bool gemm_ln_applies(const GemmArgs& a);
 et_status gemm_run(const GemmArgs& a, cudaStream_t stream);
+// FFN1 -> FFN2 in one launch when FFN1's pieces coincide with FFN2's K parts (kernels/tsgemm.cu)
+bool gemm_ffn_applies(const GemmArgs& f1, const GemmArgs& f2);
+et_status gemm_ffn_run(const GemmArgs& f1, const GemmArgs& f2, cudaStream_t stream);
 // FP32 validation build (kernels/simt32.cu): CUDA-core FP32 FMA, same arguments
 et_status gemm32_run(const GemmArgs& a, cudaStream_t stream);
 

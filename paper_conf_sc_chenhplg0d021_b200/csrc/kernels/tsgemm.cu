@@ -219,14 +219,12 @@ constexpr bool is_partial(int e) { return e == ET_EPI_F32 || e == ET_EPI_PART16;
 #define GEMM_HANDOFF_WAIT(b, ph) mbar_wait_warp((b), (ph))
 #endif
 
+// One GEMM (a piece bx of token block by, K part bz) on a CTA whose TMEM is allocated (bar.tmem_base):
+// the kernel below runs one; tsgemm_ffn_kernel runs FFN1 piece c and then FFN2 K part c of the same
+// token block in one CTA.  Ends with every store of the GEMM complete and a CTA barrier.
 template <int kEpi, bool kBF16>
-__global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
-                                                             const __grid_constant__ CUtensorMap tmap_y,
-                                                             const __grid_constant__ Params p) {
-  extern __shared__ uint8_t smem_raw[];
-  // 1024-byte aligned, derived from smem_raw by pointer arithmetic so the compiler keeps the shared
-  // address space (an integer round trip would turn every access into a generic LD/ST)
-  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+__device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUtensorMap& tmap_y, const Params& p,
+                                          const int bx, const int by, const int bz, uint8_t* smem) {
   uint8_t* ring = smem;
   using SM = Smem<kEpi>;
   constexpr int kSlots = SM::kSlots;
@@ -239,12 +237,12 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   constexpr int kAPW = kAcc / kMmaWarps;   // accumulators per MMA warp
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  const Piece pc = p.piece[blockIdx.x];
+  const Piece pc = p.piece[bx];
   const bool two = pc.seg1 != pc.seg;
   const SegDev& sa = p.seg[pc.seg];
   const SegDev& sb = p.seg[pc.seg1];
-  const int m0 = blockIdx.y * 128;
-  const int z = blockIdx.z;
+  const int m0 = by * 128;
+  const int z = bz;
   const int nk = min(p.Kp, p.K - z * p.Kp) / 64;   // A chunks (64 K each) of this K part
   const int rowsA = (two ? sa.tile_rows : pc.i1) - pc.i0, rowsB = two ? pc.i1 : 0;
   const int32_t* rpa = sa.prp + (size_t)z * sa.rp_stride;
@@ -261,7 +259,7 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   // ET_GEMM_A_ROT: rotate the order per piece instead (CTAs of one token block start a quarter of
   // the block apart) — measured no faster: the L2 serves the sharing CTAs well (profiles/r01).
 #ifdef ET_GEMM_A_ROT
-  const int a_rot = (blockIdx.x & 3) * (nk >> 2);
+  const int a_rot = (bx & 3) * (nk >> 2);
 #else
   constexpr int a_rot = 0;
 #endif
@@ -312,7 +310,6 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
     for (int i = 0; i < kMaxRows / 64; ++i) bar.pair_done[i] = 0u;
     fence_mbar_init();
   }
-  if (warp == kWarpP) tmem_alloc<512>(&bar.tmem_base);
   // stage the per-CTA row pointers once (static weight metadata, not written by any predecessor, so
   // this overlaps the previous kernel's tail under PDL).  Everything the predecessor produces (A,
   // and a bias it may have computed) is read only after pdl_wait(): by the producer before its
@@ -420,7 +417,9 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
     const int kbase = z * 48;   // first tile column of this K part
     int cur_chunk = -1;         // tile chunk whose full barrier was last waited
     // one wait for the whole A block (a wait on a completed mbarrier still costs ~100-300 cycles
-    // of this warp's issue: per-chunk waits made the first round 2-3x slower than the others)
+    // of this warp's issue: per-chunk waits made the first round 2-3x slower than the others; round 2
+    // re-measured lazy per-chunk spin waits - MMAs issued while the A block still arrives - at +0.9 us
+    // per GEMM, profiles/r02/ab_gemm_a_progressive.txt: the MMA warps are also fill warps)
     mbar_wait_warp(&bar.a_all, 0);
     tc_fence_after();
     for (int kk = 0; kk < nrounds * kAPW; ++kk) {
@@ -771,10 +770,59 @@ __global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const _
   if (threadIdx.x == 0 && cta_lin < 2048) g_cta_span[cta_lin][1] = globaltimer_ns();
 #endif
   trace_cta_end(p.ts);
-  if (warp == kWarpP) {
+}
+
+template <int kEpi, bool kBF16>
+__global__ void __launch_bounds__(Roles<kEpi>::threads, 1) tsgemm_kernel(const __grid_constant__ CUtensorMap tmap_x,
+                                                             const __grid_constant__ CUtensorMap tmap_y,
+                                                             const __grid_constant__ Params p) {
+  extern __shared__ uint8_t smem_raw[];
+  // 1024-byte aligned, derived from smem_raw by pointer arithmetic so the compiler keeps the shared
+  // address space (an integer round trip would turn every access into a generic LD/ST)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  Barriers& bar = *reinterpret_cast<Barriers*>(smem + Smem<kEpi>::kRing + Smem<kEpi>::kStage);
+  const int warp = threadIdx.x >> 5;
+  if (warp == Roles<kEpi>::WP) tmem_alloc<512>(&bar.tmem_base);   // published by gemm_body's first barrier
+  gemm_body<kEpi, kBF16>(tmap_x, tmap_y, p, blockIdx.x, blockIdx.y, blockIdx.z, smem);
+  if (warp == Roles<kEpi>::WP) {
     __syncwarp();
     tc_fence_after();
-    tmem_dealloc<512>(tbase);   // .sync.aligned: the whole warp, converged
+    tmem_dealloc<512>(bar.tmem_base);   // .sync.aligned: the whole warp, converged
+  }
+}
+
+// FFN1 -> FFN2 in one CTA (NEXT-4's FFN fusion without a cross-CTA exchange): FFN1's piece c of a
+// token block is the tile-row range [48c, 48c + 48) of W_1, i.e. exactly the 768 U columns that form
+// FFN2's K part c, so the CTA that produced them runs FFN2's K part c next.  U still goes through L2
+// (the CTA's own TMA stores, complete at the end of phase 1, read back by phase 2's TMA loads), but the
+// FFN2 kernel boundary - launch, prologue, the wait for FFN1's slowest CTA - disappears.
+template <int kEpi1, int kEpi2, bool kBF16>
+__global__ void __launch_bounds__(Roles<kEpi1>::threads, 1) tsgemm_ffn_kernel(const __grid_constant__ CUtensorMap tmx1,
+                                                                  const __grid_constant__ CUtensorMap tmy1,
+                                                                  const __grid_constant__ CUtensorMap tmx2,
+                                                                  const __grid_constant__ CUtensorMap tmy2,
+                                                                  const __grid_constant__ Params p1,
+                                                                  const __grid_constant__ Params p2) {
+  static_assert(Smem<kEpi1>::kRing == Smem<kEpi2>::kRing && Smem<kEpi1>::kStage == Smem<kEpi2>::kStage,
+                "both phases share one shared-memory layout");
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  Barriers& bar = *reinterpret_cast<Barriers*>(smem + Smem<kEpi1>::kRing + Smem<kEpi1>::kStage);
+  const int warp = threadIdx.x >> 5;
+  if (warp == Roles<kEpi1>::WP) tmem_alloc<512>(&bar.tmem_base);
+  gemm_body<kEpi1, kBF16>(tmx1, tmy1, p1, blockIdx.x, blockIdx.y, 0, smem);
+  // phase 1's U stores are complete (bulk wait + barrier at the end of gemm_body); order them before
+  // phase 2's loads of the same bytes, and every phase-1 tcgen05 op before phase 2 refills TMEM
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+  __threadfence();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  gemm_body<kEpi2, kBF16>(tmx2, tmy2, p2, 0, blockIdx.y, blockIdx.x, smem);
+  if (warp == Roles<kEpi1>::WP) {
+    __syncwarp();
+    tc_fence_after();
+    tmem_dealloc<512>(bar.tmem_base);
   }
 }
 
@@ -914,8 +962,12 @@ static int ln_pieces(const GemmArgs& a) {
 
 bool gemm_ln_applies(const GemmArgs& a) { return ln_pieces(a) > 0; }
 
-et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
-  if (a.dtype == ET_FP32) return gemm32_run(a, stream);   // FP32 validation build (CUDA cores)
+// Launch plan of one tile GEMM: parameters, tensor maps and grid.  force_pieces > 0 replaces the
+// piece planner with that many equal tile-row pieces of the (single) segment (the FFN fusion needs
+// FFN1's pieces to coincide with FFN2's K parts).  *np_out = 0: nothing to launch (M == 0).
+static et_status build_gemm(const GemmArgs& a, Params& prm, CUtensorMap& tm, CUtensorMap& tmy, dim3& grid,
+                            int force_pieces, int* np_out) {
+  *np_out = 0;
   if (a.K % 64) return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K must be a multiple of 64 (got %d)", a.K);
   if (!aligned16(a.X) || (a.ldx * 2) % 16 || (a.k0 * 2) % 16)
     return fail(ET_ERR_INVALID_ARG, "tile GEMM: X must be 16-byte aligned with 16-byte row pitch");
@@ -927,7 +979,7 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K > 768 needs a partial-sum (split-K) epilogue");
   if (a.M <= 0) return ET_OK;
 
-  Params prm{};
+  prm = Params{};
   prm.M = a.M;
   prm.K = a.K;
   prm.box_rows = a.M < 128 ? a.M : 128;
@@ -1005,7 +1057,19 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     }
     if (!ok) contiguous = false;
   }
-  if (ln) {
+  if (force_pieces > 0) {
+    if (a.nseg != 1 || a.seg[0].tile_rows % force_pieces || force_pieces > kMaxPieces ||
+        !fits(a.seg[0].tile_rows / force_pieces))
+      return fail(ET_ERR_INTERNAL, "tile GEMM: forced piece plan does not fit");
+    const int R = a.seg[0].tile_rows / force_pieces;
+    np = 0;
+    for (int k = 0; k < force_pieces; ++k) {
+      prm.piece[np].seg = prm.piece[np].seg1 = 0;
+      prm.piece[np].i0 = (int16_t)(k * R);
+      prm.piece[np].i1 = (int16_t)((k + 1) * R);
+      ++np;
+    }
+  } else if (ln) {
     const int R = a.seg[0].tile_rows / ln_np;
     for (int k = 0; k < ln_np; ++k) {
       prm.piece[np].seg = prm.piece[np].seg1 = 0;
@@ -1041,12 +1105,11 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     }
   }
   prm.npieces = np;
-  CUtensorMap tm;   // the K offset k0 is folded into the base address
+  // the K offset k0 is folded into the base address
   ET_TRY(make_tmap_2d(&tm, static_cast<const uint8_t*>(a.X) + (size_t)a.k0 * 2, a.dtype, (uint64_t)a.M,
                       (uint64_t)a.K, (uint64_t)a.ldx, 64, (uint32_t)prm.box_rows, true));
   // output tensor map: [M, ldy] in the operand dtype, box 32 cols x 32 rows (one epilogue warp's
   // staging tile, SWIZZLE_64B); fp32 partials: [kparts, M, ldy], box 32 x 32 x 1 (SWIZZLE_128B).
-  CUtensorMap tmy;
   if (a.epi == ET_EPI_F32 || a.epi == ET_EPI_PART16) {
     ET_TRY(make_tmap_3d(&tmy, a.Y, a.epi == ET_EPI_F32 ? ET_FP32 : a.dtype, (uint64_t)a.ldy, (uint64_t)a.M,
                         (uint64_t)kparts, 32, a.M < 32 ? (uint32_t)a.M : 32u));
@@ -1054,7 +1117,21 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     ET_TRY(make_tmap_2d_sw64(&tmy, a.Y, a.dtype, (uint64_t)a.M, (uint64_t)a.ldy, (uint64_t)a.ldy, 32,
                              a.M < 32 ? (uint32_t)a.M : 32u));
   }
-  dim3 grid(np, mblocks, kparts);
+  grid = dim3(np, mblocks, kparts);
+  *np_out = np;
+  return ET_OK;
+}
+
+et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
+  if (a.dtype == ET_FP32) return gemm32_run(a, stream);   // FP32 validation build (CUDA cores)
+  Params prm;
+  CUtensorMap tm, tmy;
+  dim3 grid;
+  int np = 0;
+  ET_TRY(build_gemm(a, prm, tm, tmy, grid, 0, &np));
+  if (np == 0) return ET_OK;
+  const bool ln = a.epi == (et_epilogue)kEpiLN;
+  const int ln_np = ln ? ln_pieces(a) : 0;
   const bool bf = a.dtype == ET_BF16;
   switch ((int)a.epi) {
     case ET_EPI_BIAS: return bf ? launch_typed<ET_EPI_BIAS, true>(tm, tmy, prm, grid, stream)
@@ -1074,6 +1151,49 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
     default: break;
   }
   return fail(ET_ERR_INVALID_ARG, "tile GEMM: bad epilogue %d", (int)a.epi);
+}
+
+// FFN1 -> FFN2 in one launch (tsgemm_ffn_kernel).  Applies when FFN1 has one segment with K <= 768
+// and a 16-bit bias + activation epilogue, FFN2 writes 16-bit split-K partial planes over K = FFN1's
+// output width, and FFN1 split into FFN2's K parts (768 output columns = 48 tile rows each) fills one
+// wave of the GPU with every CTA holding a full 48-row piece (C3: 4 pieces x 32 token blocks).
+bool gemm_ffn_applies(const GemmArgs& f1, const GemmArgs& f2) {
+  if (f1.dtype == ET_FP32 || f1.dtype != f2.dtype || f1.nseg != 1 || f2.nseg != 1 || f1.M != f2.M) return false;
+  if (f1.K > 768 || (f1.epi != ET_EPI_BIAS_GELU && f1.epi != ET_EPI_BIAS_RELU) || f2.epi != ET_EPI_PART16) return false;
+  if (f2.X != f1.Y || f2.ldx != f1.ldy || f2.k0 != 0 || f2.K != f1.seg[0].tile_rows * 16 || f2.K % 768) return false;
+  const int kparts = f2.K / 768, mblocks = (f1.M + 127) / 128;
+  return kparts * mblocks <= 148 && kparts * mblocks >= 96 && f1.seg[0].tile_rows == kparts * 48;
+}
+
+et_status gemm_ffn_run(const GemmArgs& f1, const GemmArgs& f2, cudaStream_t stream) {
+  if (!gemm_ffn_applies(f1, f2)) return fail(ET_ERR_INTERNAL, "FFN fusion does not apply");
+  Params p1, p2;
+  CUtensorMap tx1, ty1, tx2, ty2;
+  dim3 g1, g2;
+  int np1 = 0, np2 = 0;
+  ET_TRY(build_gemm(f1, p1, tx1, ty1, g1, f2.K / 768, &np1));
+  ET_TRY(build_gemm(f2, p2, tx2, ty2, g2, 1, &np2));
+  if (np1 == 0) return ET_OK;
+  if ((int)g1.x != (int)g2.z || g1.y != g2.y || g2.x != 1) return fail(ET_ERR_INTERNAL, "FFN fusion: plans differ");
+  const bool bf = f1.dtype == ET_BF16;
+  auto go = [&](auto kern) -> et_status {
+    static std::once_flag once;
+    static cudaError_t attr_err = cudaSuccess;
+    std::call_once(once, [&] {
+      attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)Smem<ET_EPI_PART16>::kBytes);
+    });
+    ET_CUDA(attr_err);
+    ET_CUDA(launch_pdl(kern, g1, dim3(Roles<ET_EPI_PART16>::threads), Smem<ET_EPI_PART16>::kBytes, stream, tx1, ty1,
+                       tx2, ty2, p1, p2));
+    count_launch();
+    return ET_OK;
+  };
+  if (f1.epi == ET_EPI_BIAS_GELU)
+    return bf ? go(tsgemm_ffn_kernel<ET_EPI_BIAS_GELU, ET_EPI_PART16, true>)
+              : go(tsgemm_ffn_kernel<ET_EPI_BIAS_GELU, ET_EPI_PART16, false>);
+  return bf ? go(tsgemm_ffn_kernel<ET_EPI_BIAS_RELU, ET_EPI_PART16, true>)
+            : go(tsgemm_ffn_kernel<ET_EPI_BIAS_RELU, ET_EPI_PART16, false>);
 }
 
 #ifdef ET_TIMELINE
