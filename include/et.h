@@ -292,12 +292,29 @@ et_status et_attention_pre_fwd(const et_attn_desc* desc, const void* X, const et
                                const float* ln_gamma, const float* ln_beta, float ln_eps, void* out, void* workspace,
                                size_t ws_bytes, void* stream);
 
-/* One encoder layer's parameters.  Weights packed; biases in the storage dtype; LN fp32. */
+/* One encoder layer's parameters.  Weights packed; biases in the storage dtype; LN fp32.
+ * Attention-aware layers (row-pruned W_V, PAPER.md line 107 / 317) may carry the layer data that
+ * depends only on the weights, computed once by et_vprep: v_col / v_width [heads] (each head's packed
+ * V columns), bv_packed [wv.rows_padded] (b_V of the kept rows, 0 in padding rows) and bo_folded [d]
+ * (b_O' = b_O + sum over pruned V features f of W_O'[:, f] b_V[f], reading C-6), all device memory
+ * in the storage dtype (int32 for the column tables).  All four NULL (or a tile-pruned W_V): the
+ * forward computes them on its stream every call (three extra launches per layer). */
 typedef struct {
   et_packed_weight wq, wk, wv, wo, w1, w2;
   const void *bq, *bk, *bv, *bo, *b1, *b2;
   const float *ln1_g, *ln1_b, *ln2_g, *ln2_b;
+  const int32_t *v_col, *v_width;
+  const void *bv_packed, *bo_folded;
 } et_layer;
+
+/* et_vprep: the attention-aware layer data of et_layer (above) for a row-pruned W_V (packed with
+ * group_rows = d_model / heads) and its W_O; bv / bo [d] in dtype (bo may be NULL: b_O' is then the
+ * fold alone).  Outputs caller-allocated device memory: v_col, v_width [heads] int32, bv_packed
+ * [wv->rows_padded] and bo_folded [d_model] in dtype.  Stream-ordered; ET_ERR_INVALID_ARG for a
+ * tile-pruned W_V or mismatched shapes. */
+et_status et_vprep(const et_packed_weight* wv, const et_packed_weight* wo, const void* bv, const void* bo,
+                   int32_t heads, int32_t d_model, et_dtype dtype, int32_t* v_col, int32_t* v_width,
+                   void* bv_packed, void* bo_folded, void* stream);
 
 /* Post-LN encoder stack:  for each layer:
  *   Y1 = LN(X + SelfAttn(X));  U = act(Y1 W1'^T + b1);  Y2 = LN(Y1 + U W2'^T + b2).

@@ -64,7 +64,8 @@ class AttnDescC(ctypes.Structure):
 class LayerC(ctypes.Structure):
     _fields_ = [("wq", PackedWeightC), ("wk", PackedWeightC), ("wv", PackedWeightC), ("wo", PackedWeightC),
                 ("w1", PackedWeightC), ("w2", PackedWeightC), ("bq", _vp), ("bk", _vp), ("bv", _vp), ("bo", _vp),
-                ("b1", _vp), ("b2", _vp), ("ln1_g", _vp), ("ln1_b", _vp), ("ln2_g", _vp), ("ln2_b", _vp)]
+                ("b1", _vp), ("b2", _vp), ("ln1_g", _vp), ("ln1_b", _vp), ("ln2_g", _vp), ("ln2_b", _vp),
+                ("v_col", _vp), ("v_width", _vp), ("bv_packed", _vp), ("bo_folded", _vp)]
 
 
 def _sig(name, res, args):
@@ -366,13 +367,38 @@ class Layer:
             setattr(c, n, packed[n].c)
         for n in ("bq", "bk", "bv", "bo", "b1", "b2", "ln1_g", "ln1_b", "ln2_g", "ln2_b"):
             setattr(c, n, dense[n].data_ptr())
+        for n in ("v_col", "v_width", "bv_packed", "bo_folded"):   # et_vprep output (attention-aware), optional
+            setattr(c, n, dense[n].data_ptr() if n in dense else None)
         self.c = c
 
 
-def pack_layer(raw: dict, scheme: str, ratio: float, heads: int, dtype="fp16", stream=None) -> Layer:
+_vprep = _sig("et_vprep", ctypes.c_int,
+              [ctypes.POINTER(PackedWeightC), ctypes.POINTER(PackedWeightC), _vp, _vp, _i32, _i32, ctypes.c_int,
+               _vp, _vp, _vp, _vp, _vp])
+SYMBOLS += ["et_vprep"]
+
+
+def vprep(wv: "Packed", wo: "Packed", bv: torch.Tensor, bo: torch.Tensor | None, heads: int, d_model: int,
+          dtype="fp16", stream=None) -> dict:
+    """et_vprep: an attention-aware layer's weight-only data (per-head packed V columns / widths, packed
+    b_V, folded b_O'), computed once instead of on every forward."""
+    tdt = torch_dtype(dtype)
+    out = {"v_col": torch.empty(heads, dtype=torch.int32, device="cuda"),
+           "v_width": torch.empty(heads, dtype=torch.int32, device="cuda"),
+           "bv_packed": torch.empty(max(wv.c.rows_padded, 1), dtype=tdt, device="cuda"),
+           "bo_folded": torch.empty(d_model, dtype=tdt, device="cuda")}
+    _check(_vprep(ctypes.byref(wv.c), ctypes.byref(wo.c), bv.data_ptr(), _ptr(bo), heads, d_model, dtype_code(dtype),
+                  out["v_col"].data_ptr(), out["v_width"].data_ptr(), out["bv_packed"].data_ptr(),
+                  out["bo_folded"].data_ptr(), _stream(stream)))
+    return out
+
+
+def pack_layer(raw: dict, scheme: str, ratio: float, heads: int, dtype="fp16", stream=None, precompute=True) -> Layer:
     """Prune + pack the six matrices of one layer (pattern per scheme: PAPER.md line 107, 317).
 
-    raw: name -> float32 numpy/torch array holding storage-dtype values (et_synth.make_layer)."""
+    raw: name -> float32 numpy/torch array holding storage-dtype values (et_synth.make_layer).
+    precompute: for a row-pruned W_V, compute the attention-aware layer data once (et_vprep) so the
+    forward skips it; False leaves it to every forward (both paths are tested)."""
     tdt = torch_dtype(dtype)
     dev = torch.device("cuda")
     packed, dense = {}, {}
@@ -391,6 +417,8 @@ def pack_layer(raw: dict, scheme: str, ratio: float, heads: int, dtype="fp16", s
         dense[n] = torch.as_tensor(raw[n]).to(dev).to(tdt).contiguous()
     for n in ("ln1_g", "ln1_b", "ln2_g", "ln2_b"):
         dense[n] = torch.as_tensor(raw[n]).to(dev).to(torch.float32).contiguous()
+    if precompute and packed["wv"].c.pattern == PRUNE_ROW and dtype in ("fp16", "bf16"):
+        dense.update(vprep(packed["wv"], packed["wo"], dense["bv"], dense["bo"], heads, d_model, dtype, stream))
     return Layer(packed, dense)
 
 

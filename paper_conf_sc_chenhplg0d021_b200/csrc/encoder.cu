@@ -202,7 +202,8 @@ struct LnFuse {
 et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et_packed_weight* wq,
                               const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
                               const void* bq, const void* bk, const void* bv, const void* bo, const BlockWs& ws,
-                              const void** bo_eff, cudaStream_t st, LnFuse* lnf = nullptr) {
+                              const void** bo_eff, cudaStream_t st, LnFuse* lnf = nullptr,
+                              const et_layer* pre = nullptr) {
   const int dm = d->d_model, dk = dm / d->heads;
   const bool hp = head_parallel(d);
   const int Hr = d->head_end - d->head_begin, dq = Hr * dk;
@@ -214,7 +215,11 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   const void* bo_rank = (hp && d->head_begin != 0) ? nullptr : bo;   // b_O enters the sum once
   const void* bv_use = bv;
   *bo_eff = bo_rank;
-  if (rowv) {
+  const bool have_pre = rowv && pre && pre->v_col && pre->v_width && pre->bv_packed && pre->bo_folded && !hp;
+  if (have_pre) {   // computed once at pack time (et_vprep)
+    bv_use = pre->bv_packed;
+    *bo_eff = pre->bo_folded;
+  } else if (rowv) {
     // full weights: every head's packed V columns, and the fold over this range's features only
     VPrep vp{wv, wo, bv, bo_rank, full ? d->heads : Hr, dk, full ? h0 * dk : 0, full ? h0 * dk + dq : dq,
              d->dtype, ws.v_col, ws.v_width, ws.bv_packed, ws.bo_folded};
@@ -249,8 +254,8 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   a.q_off = 0;
   a.k_off = dq;
   a.v_off = 2 * dq;
-  a.v_col = rowv ? ws.v_col + (full ? h0 : 0) : nullptr;
-  a.v_width = rowv ? ws.v_width + (full ? h0 : 0) : nullptr;
+  a.v_col = have_pre ? pre->v_col : rowv ? ws.v_col + (full ? h0 : 0) : nullptr;
+  a.v_width = have_pre ? pre->v_width : rowv ? ws.v_width + (full ? h0 : 0) : nullptr;
   a.Z = ws.z;
   a.ld_z = dq;
   a.z_map = rowv ? wv->row_map : nullptr;
@@ -545,6 +550,21 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   return ET_OK;
 }
 
+et_status et_vprep(const et_packed_weight* wv, const et_packed_weight* wo, const void* bv, const void* bo,
+                   int32_t heads, int32_t d_model, et_dtype dtype, int32_t* v_col, int32_t* v_width,
+                   void* bv_packed, void* bo_folded, void* stream) {
+  if (!wv || !wo || !bv || !v_col || !v_width || !bv_packed || !bo_folded || heads <= 0 || d_model <= 0 ||
+      d_model % heads)
+    return fail(ET_ERR_INVALID_ARG, "et_vprep: null pointer or bad shape");
+  if (dtype != ET_FP16 && dtype != ET_BF16) return fail(ET_ERR_UNSUPPORTED, "et_vprep: FP16 / BF16 layers only");
+  const int dk = d_model / heads;
+  ET_TRY(check_weight(wv, d_model, d_model, dtype, "W_V", true, dk));
+  ET_TRY(check_weight(wo, d_model, d_model, dtype, "W_O", false));
+  if (wv->pattern != ET_PRUNE_ROW) return fail(ET_ERR_INVALID_ARG, "et_vprep: W_V is not row-pruned");
+  VPrep vp{wv, wo, bv, bo, heads, dk, 0, d_model, dtype, v_col, v_width, bv_packed, bo_folded};
+  return vprep_run(vp, static_cast<cudaStream_t>(stream));
+}
+
 et_status et_encoder_workspace_size(const et_attn_desc* desc, int32_t num_layers, int32_t d_ff,
                                     et_dtype resid_dtype, const et_layer* layers, size_t* bytes) {
   ET_TRY(check_desc(desc));
@@ -628,7 +648,7 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     const void* bo_eff = L.bo;
     LnFuse lf{cur_res, L.ln1_g, L.ln1_b, ln_eps, y1a, false};   // (only with the residual in the operand dtype)
     ET_TRY(run_attention_block(desc, cur_act, &L.wq, &L.wk, &L.wv, &L.wo, L.bq, L.bk, L.bv, L.bo, ws, &bo_eff, st,
-                               split ? nullptr : &lf));
+                               split ? nullptr : &lf, &L));
     // 4. Y1 = LN(X + attn) (unless fused into the O-projection above)
     if (!lf.done) {
       LnArgs ln1{ws.part, L.wo.kparts, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,

@@ -246,3 +246,24 @@ def test_attention_aware_fully_pruned_head(etm):
     Y, _, _ = _gpu(etm, cfg, raws, X, lens)
     ref = _oracle(cfg, raws, X, lens)
     assert_close(Y.reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what="C4 with an empty V head")
+
+
+@pytest.mark.parametrize("key,kw", [("C2", {}), ("C4", {"layers": 2, "batch": 2})])
+def test_vprep_at_pack_time_bitexact(etm, key, kw):
+    """Attention-aware layers: the weight-only data (per-head packed V columns / widths, packed b_V,
+    folded b_O', reading C-6) computed once at pack time by et_vprep gives the same bits as the
+    forward computing it on every call (et_layer fields NULL)."""
+    cfg, raws, X, lens = _case(key, **kw)
+    L = torch.from_numpy(lens).cuda()
+    outs = []
+    for pre in (True, False):
+        layers = [etm.pack_layer(r, cfg.scheme, cfg.ratio, cfg.heads, cfg.dtype, precompute=pre) for r in raws]
+        assert (layers[0].c.bo_folded is not None) == pre
+        enc = etm.Encoder(layers, cfg.batch, cfg.seq_len, cfg.heads, cfg.d_ff, act=cfg.act, ln_eps=cfg.ln_eps,
+                          dtype=cfg.dtype, resid_dtype=cfg.dtype, causal=cfg.causal, lengths=L)
+        n0 = etm._lib.et_launch_count()
+        outs.append(to64(enc(dev_tensor(X.reshape(cfg.tokens, cfg.d_model), cfg.dtype))))
+        torch.cuda.synchronize()
+        outs[-1] = (outs[-1], etm._lib.et_launch_count() - n0)
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert outs[0][1] + 3 * cfg.layers == outs[1][1]   # three V-prep launches per layer saved
