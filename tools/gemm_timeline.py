@@ -9,7 +9,7 @@ from et_synth import CONFIGS, make_layer
 cfg = CONFIGS["C3"]
 raw = make_layer(cfg, 0)
 lay = et.pack_layer(raw, "tile", 0.8, 12, "fp16")
-M = 4096
+M = int(sys.argv[1]) if len(sys.argv) > 1 else 4096
 X = torch.randn(M, 768, device='cuda').half()
 U = torch.randn(M, 3072, device='cuda').half()
 buf = (ctypes.c_ulonglong * 512)()
