@@ -267,3 +267,16 @@ def test_vprep_at_pack_time_bitexact(etm, key, kw):
         outs[-1] = (outs[-1], etm._lib.et_launch_count() - n0)
     assert np.array_equal(outs[0][0], outs[1][0])
     assert outs[0][1] + 3 * cfg.layers == outs[1][1]   # three V-prep launches per layer saved
+
+
+def test_fused_ffn_ragged_token_blocks(etm):
+    """The one-launch FFN1 -> FFN2 path (tsgemm_ffn_kernel) with a ragged last token block: 24
+    sequences of 125 tokens = 3000 rows = 23 full blocks + 56 rows, 24 x 4 = 96 CTAs (the fused path
+    applies between 96 and 148 CTAs); two layers against the oracle on sampled sequences, the last
+    one inside the ragged block."""
+    cfg, raws, X, lens = _case("C3", layers=2, batch=24, seq_len=125)
+    assert (cfg.tokens + 127) // 128 * 4 >= 96
+    Y, _, _ = _gpu(etm, cfg, raws, X, lens)
+    idx = np.array([0, 1, 23])
+    ref = _oracle(cfg, raws, X, lens, idx)
+    assert_close(Y[idx].reshape(-1, cfg.d_model), ref.reshape(-1, cfg.d_model), what="C3 ragged fused FFN")
