@@ -232,6 +232,7 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
   Barriers& bar = *reinterpret_cast<Barriers*>(smem + SM::kRing + SM::kStage);
 
   constexpr bool kLN = kEpi == kEpiLN;
+
   constexpr int kMmaWarps = Roles<kEpi>::MW, kEpiGroups = Roles<kEpi>::EG, kEpiWarps = Roles<kEpi>::EW;
   constexpr int kWarpP = Roles<kEpi>::WP, kFillSets = kWarpP / 4, kThreads = Roles<kEpi>::threads;
   constexpr int kAPW = kAcc / kMmaWarps;   // accumulators per MMA warp
@@ -305,7 +306,8 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
     if (nchunks > kMaxBChunks || nrows > kMaxRows || (!is_partial(kEpi) && nrows > kMaxBiasRows))
       __trap();   // host sizes pieces so this cannot happen
     for (int i = 0; i < kAcc; ++i) mbar_init(&bar.acc_empty[i], 4);
-    for (int j = 0; j < npairs_all; ++j) mbar_init(&bar.slot_full[j], min(2, nrows - 2 * j));   // one commit per row
+    for (int j = 0; j < npairs_all; ++j)   // one commit per row (MMA warps) or per pair (epilogue-issued)
+      mbar_init(&bar.slot_full[j], min(2, nrows - 2 * j));
     for (int i = 0; i < nchunks; ++i) mbar_init(&bar.bfull[i], 1);
     for (int i = 0; i < kMaxRows / 64; ++i) bar.pair_done[i] = 0u;
     fence_mbar_init();
@@ -327,6 +329,60 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
   if constexpr (kLN) cluster_arrive_relaxed();   // phase A: this CTA runs (DSMEM targets exist)
   // end of local row t's tiles (part A's last row ends before the padding to part B's first chunk)
   auto rend = [&](int t) { return t == rowsA - 1 ? min(bar.a_end, bar.rptr[t + 1]) : bar.rptr[t + 1]; };
+
+  // One tile row's MMA chain into accumulator `acc` (warp-collective; one elected lane issues).  The
+  // row's tiles lie in chunks [q0 / 32, (q1 - 1) / 32]; a segment = the row's tiles inside one chunk:
+  // wait for the chunk once, read the tile columns lane-parallel, issue the MMAs from register
+  // broadcasts.  The first segment is prepared BEFORE `before_issue` (the accumulator hand-off), so
+  // the barrier / shared-memory / shuffle latency stays off the accumulator's critical path.
+  const uint32_t idesc = make_idesc_f16(128, 16, kBF16 ? 1 : 0, 0, 0);
+  const uint32_t ring_u32 = smem_u32(ring);
+  const int kbase = z * 48;   // first tile column of this K part
+  auto issue_row = [&](int t, int acc, int k, int& cur_chunk, auto&& before_issue) {
+    const uint32_t d_tmem = tbase + kAccCol + acc * 16;
+    const int q0 = bar.rptr[t], q1 = rend(t);   // this row's tiles, relative to the CTA's stream
+    int qb = q0, qe = q0, n = 0, mycol = 0;
+    uint32_t acol = 0, blo = 0, bhi = 0;
+    auto prep = [&]() {
+      const int c = qb / kChunkTiles;
+      qe = min(q1, (c + 1) * kChunkTiles);
+      if (c != cur_chunk) {
+        mbar_wait_warp(&bar.bfull[c], 0);
+        if (lane == 0 && c < 40) ET_TL_MIN(400 + c);   // first time any issuer saw tile chunk c (debug)
+        cur_chunk = c;
+        tc_fence_after();
+      }
+      const int slot = pos_t(c) % kSlots;
+      const int coff = two ? bar.tcoff[slot] : (pbA + c * kChunkTiles) & 3;
+      n = qe - qb;
+      mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
+      // B descriptor of tile u: start address field advances by 512 B / 16 = 32 per tile
+      const uint64_t bd0 = make_sdesc(ring_u32 + slot * kSlotBytes + (qb % kChunkTiles) * 512, 128, 256,
+                                      kLayoutNone);
+      blo = (uint32_t)bd0;
+      bhi = (uint32_t)(bd0 >> 32);
+      acol = tbase + (uint32_t)(mycol * 8);   // this lane's tile: its A columns
+    };
+    if (qb < q1) prep();
+    before_issue();
+    if (lane == 0 && warp < kMmaWarps && k < 8) ET_TL(16 + 24 * warp + 3 * k);
+    while (qb < q1) {
+      int u = 0;
+      for (; u + 4 <= n; u += 4) {
+        if (lane == 0 && warp < kMmaWarps && k < 8 && qb + u == q0) ET_TL(16 + 24 * warp + 3 * k + 1);
+        mma_ts_warp_x4(d_tmem, __shfl_sync(0xffffffffu, acol, u), __shfl_sync(0xffffffffu, acol, u + 1),
+                       __shfl_sync(0xffffffffu, acol, u + 2), __shfl_sync(0xffffffffu, acol, u + 3),
+                       blo + 32 * u, blo + 32 * (u + 1), blo + 32 * (u + 2), blo + 32 * (u + 3), bhi, idesc,
+                       (qb + u) != q0);
+      }
+      for (; u < n; ++u) {
+        const uint32_t a = __shfl_sync(0xffffffffu, acol, u);
+        mma_ts_warp_nc(d_tmem, a, ((uint64_t)bhi << 32) | (blo + 32 * u), idesc, (qb + u) != q0);
+      }
+      qb = qe;
+      if (qb < q1) prep();
+    }
+  };
 
   if (warp < kWarpP) {
     // A fill, smem ring -> TMEM through registers: chunk j is moved by the four warps of set j % 6,
@@ -412,73 +468,32 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
     }
   } else if (warp < kMmaWarps) {
     // ===================== MMA warps: warp w issues the chains of tile rows w, w+8, w+16, ...
-    const uint32_t idesc = make_idesc_f16(128, 16, kBF16 ? 1 : 0, 0, 0);
-    const uint32_t ring_u32 = smem_u32(ring);
-    const int kbase = z * 48;   // first tile column of this K part
-    int cur_chunk = -1;         // tile chunk whose full barrier was last waited
-    // one wait for the whole A block (a wait on a completed mbarrier still costs ~100-300 cycles
-    // of this warp's issue: per-chunk waits made the first round 2-3x slower than the others; round 2
-    // re-measured lazy per-chunk spin waits - MMAs issued while the A block still arrives - at +0.9 us
-    // per GEMM, profiles/r02/ab_gemm_a_progressive.txt: the MMA warps are also fill warps)
-    mbar_wait_warp(&bar.a_all, 0);
-    tc_fence_after();
-    for (int kk = 0; kk < nrounds * kAPW; ++kk) {
-      const int k = kk / kAPW;                     // round
-      const int acc = warp + (kk % kAPW) * kMmaWarps;   // accumulator (rows in increasing order)
-      const int t = k * kAcc + acc;
-      if (t >= nrows) break;
-      const uint32_t d_tmem = tbase + kAccCol + acc * 16;
-      const int q0 = bar.rptr[t], q1 = rend(t);   // this row's tiles, relative to the CTA's stream
-      // The row's tiles lie in chunks [q0 / 32, (q1 - 1) / 32].  A segment = the row's tiles inside
-      // one chunk: wait for the chunk once, read the tile columns lane-parallel, issue the MMAs from
-      // register broadcasts.  The first segment is prepared BEFORE waiting for the accumulator, so
-      // the barrier / shared-memory / shuffle latency stays off the accumulator's critical path.
-      int qb = q0, qe = q0, n = 0, mycol = 0;
-      uint32_t acol = 0, blo = 0, bhi = 0;
-      auto prep = [&]() {
-        const int c = qb / kChunkTiles;
-        qe = min(q1, (c + 1) * kChunkTiles);
-        if (c != cur_chunk) {
-          mbar_wait_warp(&bar.bfull[c], 0);
-          if (lane == 0 && c < 40) ET_TL_MIN(400 + c);   // first time any MMA warp saw tile chunk c (debug)
-          cur_chunk = c;
-          tc_fence_after();
-        }
-        const int slot = pos_t(c) % kSlots;
-        const int coff = two ? bar.tcoff[slot] : (pbA + c * kChunkTiles) & 3;
-        n = qe - qb;
-        mycol = lane < n ? bar.tcol[slot][coff + (qb % kChunkTiles) + lane] - kbase : 0;
-        // B descriptor of tile u: start address field advances by 512 B / 16 = 32 per tile
-        const uint64_t bd0 = make_sdesc(ring_u32 + slot * kSlotBytes + (qb % kChunkTiles) * 512, 128, 256,
-                                        kLayoutNone);
-        blo = (uint32_t)bd0;
-        bhi = (uint32_t)(bd0 >> 32);
-        acol = tbase + (uint32_t)(mycol * 8);   // this lane's tile: its A columns
-      };
-      if (qb < q1) prep();
-      if (k > 0) {   // the epilogue group must have read this accumulator's previous row
-        GEMM_HANDOFF_WAIT(&bar.acc_empty[acc], (k - 1) & 1);
-        tc_fence_after();
+    // (Round 2 measured the alternative of the epilogue groups issuing their accumulator pair's next
+    // chains right after draining it - a named barrier instead of the mbarrier hand-off: 29.1k / 34.9k
+    // seq/s with one / two issuing warps per group against 41.1k, profiles/r02/ab_gemm_epilogue_issue.txt:
+    // issue and epilogue math serialise on the same warps.)
+    {
+      int cur_chunk = -1;         // tile chunk whose full barrier was last waited
+      // one wait for the whole A block (a wait on a completed mbarrier still costs ~100-300 cycles
+      // of this warp's issue: per-chunk waits made the first round 2-3x slower than the others; round 2
+      // re-measured lazy per-chunk spin waits - MMAs issued while the A block still arrives - at +0.9 us
+      // per GEMM, profiles/r02/ab_gemm_a_progressive.txt: the MMA warps are also fill warps)
+      mbar_wait_warp(&bar.a_all, 0);
+      tc_fence_after();
+      for (int kk = 0; kk < nrounds * kAPW; ++kk) {
+        const int k = kk / kAPW;                     // round
+        const int acc = warp + (kk % kAPW) * kMmaWarps;   // accumulator (rows in increasing order)
+        const int t = k * kAcc + acc;
+        if (t >= nrows) break;
+        issue_row(t, acc, k, cur_chunk, [&]() {   // the epilogue group must have read the previous row
+          if (k > 0) {
+            GEMM_HANDOFF_WAIT(&bar.acc_empty[acc], (k - 1) & 1);
+            tc_fence_after();
+          }
+        });
+        mma_commit_warp(&bar.slot_full[t >> 1]);   // fires when this row's MMAs are complete
+        if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k + 2);
       }
-      if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k);
-      while (qb < q1) {
-        int u = 0;
-        for (; u + 4 <= n; u += 4) {
-          if (lane == 0 && k < 8 && qb + u == q0) ET_TL(16 + 24 * warp + 3 * k + 1);
-          mma_ts_warp_x4(d_tmem, __shfl_sync(0xffffffffu, acol, u), __shfl_sync(0xffffffffu, acol, u + 1),
-                         __shfl_sync(0xffffffffu, acol, u + 2), __shfl_sync(0xffffffffu, acol, u + 3),
-                         blo + 32 * u, blo + 32 * (u + 1), blo + 32 * (u + 2), blo + 32 * (u + 3), bhi, idesc,
-                         (qb + u) != q0);
-        }
-        for (; u < n; ++u) {
-          const uint32_t a = __shfl_sync(0xffffffffu, acol, u);
-          mma_ts_warp_nc(d_tmem, a, ((uint64_t)bhi << 32) | (blo + 32 * u), idesc, (qb + u) != q0);
-        }
-        qb = qe;
-        if (qb < q1) prep();
-      }
-      mma_commit_warp(&bar.slot_full[t >> 1]);   // fires when this row's MMAs are complete
-      if (lane == 0 && k < 8) ET_TL(16 + 24 * warp + 3 * k + 2);
     }
   } else {
     // ===================== epilogue warps: group g drains the accumulators of MMA warps 2g, 2g+1
@@ -534,6 +549,7 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
       if (lane == 0)
         for (int a = 0; a < na; ++a) mbar_arrive(&bar.acc_empty[pidx * 2 + a]);
       if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it + 1);
+      if (quarter > 0 && lane == 0 && it < 4 && g == 0) ET_TL(386 + 4 * (quarter - 1) + it);   // debug
       // math: bias / scale / activation on the pair's 32 columns of this thread's token row
       float v[32];
 #pragma unroll

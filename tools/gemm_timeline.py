@@ -49,3 +49,5 @@ for name, w, x, epi, b in [("wq", "wq", X, et.EPI_BIAS_SCALE, "bq"), ("ffn1", "w
     for g in range(4):
         print(f"  epi g{g}: " + " ".join("[" + ",".join(str(rel(208 + 40 * g + 5 * k + i)) for i in range(4)) + "]"
                                        for k in range(6)))
+    print("  w0/w1 next row prepared (rounds 0-7): " + " ".join(str(rel(370 + i)) for i in range(16)))
+    print("  g0 quarters 1-3 drained (rounds 0-3): " + " ".join(str(rel(386 + i)) for i in range(12)))
