@@ -265,6 +265,7 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
     if (!rowv) a.Z = static_cast<uint8_t*>(ws.z) + (size_t)h0 * dk * dtype_size(d->dtype);   // row_map is global
   }
   a.z_clear = rowv ? 1 : 0;
+  a.vtab_static = have_pre ? 1 : 0;   // et_vprep tables: readable before the grid-dependency wait
   a.lengths = d->lengths_dev;
   a.batch = d->batch;
   a.seq_len = d->seq_len;

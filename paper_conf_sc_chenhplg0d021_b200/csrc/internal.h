@@ -130,6 +130,7 @@ struct AttnArgs {
   int z_clear;              // z_map mode: Z columns no kept V feature maps to must be zero afterwards
                             // (attention_run zero-fills whole head windows or memsets Z; one place decides)
   int generic;              // force the generic short-form kernel (ET_ATTN_SHORT_GENERIC test hook)
+  int vtab_static;          // v_col / v_width are layer weights (not written by a predecessor kernel)
 };
 et_status attention_run(const AttnArgs& a, cudaStream_t stream);
 et_status attention32_run(const AttnArgs& a, cudaStream_t stream);

@@ -73,6 +73,7 @@ struct AParams {
   int tma_store;            // Z written through TMA stores (dense V layout, seq_len % 32 == 0)
   int z_stage;              // z_map scatter staged in shared memory, stored as 16-byte row windows
   int z_fill_empty;         // (with z_stage) a head with no kept V feature writes zeros over its Z window
+  int vtab_static;          // v_col / v_width are layer weights (et_vprep at pack time): read before the grid wait
   unsigned long long* ts;   // trace slot or nullptr
 };
 
@@ -111,12 +112,21 @@ __global__ void __launch_bounds__(kThreads, kLong ? 1 : 2) attn_kernel(const __g
   constexpr int kS = 0, kP = 128 * kNKB, kO = 192 * kNKB;
   constexpr uint32_t kCols = (kO + kDK) <= 256 ? 256u : 512u;
   pdl_trigger();
-  pdl_wait();   // QKV (and the attention-aware head tables) of the predecessors are visible from here
-  trace_cta_start(p.ts);
-  // attention-aware head tables: both loads issued together (one latency, not two in series)
+  // attention-aware head tables: both loads issued together (one latency, not two in series); when
+  // they are layer weights (computed at pack time) they are read before the grid-dependency wait, so
+  // their latency overlaps the predecessor instead of sitting in front of every CTA's work
   const int hh = p.head_begin + blockIdx.y;
-  const int vloc = p.v_col ? __ldg(p.v_col + hh) : hh * kDK;   // packed V column of this head
-  const int vw = p.v_width ? __ldg(p.v_width + hh) : kDK;
+  int vloc = hh * kDK, vw = kDK;
+  if (p.vtab_static) {
+    if (p.v_col) vloc = __ldg(p.v_col + hh);
+    if (p.v_width) vw = __ldg(p.v_width + hh);
+  }
+  pdl_wait();   // QKV (and per-forward head tables) of the predecessors are visible from here
+  trace_cta_start(p.ts);
+  if (!p.vtab_static) {
+    if (p.v_col) vloc = __ldg(p.v_col + hh);     // packed V column of this head
+    if (p.v_width) vw = __ldg(p.v_width + hh);
+  }
   if (vw == 0) {   // every V feature of the head pruned: Z = 0 there (reading C-6: b_V folded into b_O')
     if (p.z_fill_empty) {   // the staged path writes every other head's whole window: no Z memset needed
       using T0 = typename std::conditional<kBF16, __nv_bfloat16, __half>::type;
@@ -616,6 +626,7 @@ et_status attention_run(const AttnArgs& a, cudaStream_t stream) {
                    aligned16(a.Z) && (a.ld_z * 2) % 16 == 0) ? 1 : 0;
   prm.z_stage = z_staged(a) ? 1 : 0;
   prm.z_fill_empty = prm.z_stage && a.z_clear;
+  prm.vtab_static = a.vtab_static;
   if (prm.tma_store) {
     ET_TRY(make_tmap_2d_sw64(&tz, a.Z, a.dtype, rows, (uint64_t)a.ld_z, (uint64_t)a.ld_z, 32, 32));
   } else {
