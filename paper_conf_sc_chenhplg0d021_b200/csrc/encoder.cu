@@ -180,17 +180,6 @@ void carve_block(Carver& c, const et_attn_desc* d, int vmax, int kparts_max, Blo
   ws->splitk = kp_d > 1 ? c.take((size_t)kp_d * M * (std::max(ws->ldq, splitk_cols) + 8) * 4) : nullptr;
 }
 
-// Step 4 fused into the O-projection when possible (kEpiLN: residual in the operand dtype, full head
-// range): Y1 = LN(resid + Z W_O'^T + b_O') written straight to `out`; `done` reports whether it ran.
-struct LnFuse {
-  const void* resid;
-  const float* gamma;
-  const float* beta;
-  float eps;
-  void* out;
-  bool done;
-};
-
 // Steps 1-3 (+4 when gamma != NULL): attention block on X (act dtype), output the O-projection
 // partial in ws->part (for the caller's LayerNorm step, which adds *bo_eff).
 // Head-parallel mode (desc head range [h0, h1) != [0, H); Megatron-style split of Eq. 4,
@@ -202,8 +191,7 @@ struct LnFuse {
 et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et_packed_weight* wq,
                               const et_packed_weight* wk, const et_packed_weight* wv, const et_packed_weight* wo,
                               const void* bq, const void* bk, const void* bv, const void* bo, const BlockWs& ws,
-                              const void** bo_eff, cudaStream_t st, LnFuse* lnf = nullptr,
-                              const et_layer* pre = nullptr) {
+                              const void** bo_eff, cudaStream_t st, const et_layer* pre = nullptr) {
   const int dm = d->d_model, dk = dm / d->heads;
   const bool hp = head_parallel(d);
   const int Hr = d->head_end - d->head_begin, dq = Hr * dk;
@@ -293,21 +281,6 @@ et_status run_attention_block(const et_attn_desc* d, const void* X_act, const et
   o.Y = ws.part;
   o.ldy = dm;
   o.epi = hp ? ET_EPI_F32 : part_epi_of(d->dtype);
-  if (lnf && !hp) {   // 3+4 fused: bias, residual and LayerNorm in the GEMM epilogue (cluster DSMEM)
-    GemmArgs f = o;
-    f.seg[0] = seg_of(wo, *bo_eff, 0);
-    f.epi = (et_epilogue)kEpiLN;
-    f.Y = lnf->out;
-    f.resid = lnf->resid;
-    f.gamma = lnf->gamma;
-    f.beta = lnf->beta;
-    f.eps = lnf->eps;
-    if (gemm_ln_applies(f)) {
-      f.ts = trace_slot(ET_K_OPROJ);
-      lnf->done = true;
-      return gemm_run(f, st);
-    }
-  }
   o.ts = trace_slot(ET_K_OPROJ);
   return gemm_run(o, st);
 }
@@ -536,10 +509,7 @@ et_status et_attention_fwd(const et_attn_desc* desc, const void* X, const et_pac
   BlockWs ws;
   carve_block(c, desc, v_cols_of(wv, full ? dm : dq), 1, &ws, full);
   const void* bo_eff = bo;
-  LnFuse lf{X, ln_gamma, ln_beta, ln_eps, out, false};
-  ET_TRY(run_attention_block(desc, X, wq, wk, wv, wo, bq, bk, bv, bo, ws, &bo_eff, st,
-                             (ln_gamma && !hp) ? &lf : nullptr));
-  if (lf.done) return ET_OK;
+  ET_TRY(run_attention_block(desc, X, wq, wk, wv, wo, bq, bk, bv, bo, ws, &bo_eff, st));
   const int M = desc->batch * desc->seq_len;
   // full range: out = part + b_O' (+ X and LN when gamma is given), in dtype;
   // head-parallel: out = FP32 partial (+ b_O' on the rank owning head 0), no residual / LN
@@ -647,16 +617,13 @@ et_status et_encoder_fwd(const et_attn_desc* desc, int32_t num_layers, int32_t d
     void* next_res = ((num_layers - 1 - l) % 2 == 0) ? out : tmp_res;
     void* next_act = split ? xa : next_res;
     const void* bo_eff = L.bo;
-    LnFuse lf{cur_res, L.ln1_g, L.ln1_b, ln_eps, y1a, false};   // (only with the residual in the operand dtype)
     ET_TRY(run_attention_block(desc, cur_act, &L.wq, &L.wk, &L.wv, &L.wo, L.bq, L.bk, L.bv, L.bo, ws, &bo_eff, st,
-                               split ? nullptr : &lf, &L));
-    // 4. Y1 = LN(X + attn) (unless fused into the O-projection above)
-    if (!lf.done) {
-      LnArgs ln1{ws.part, L.wo.kparts, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,
-                 y1a, split ? y1r : nullptr, nullptr, part_dtype_of(desc->dtype)};
-      ln1.ts = trace_slot(ET_K_LN1);
-      ET_TRY(layernorm_run(ln1, st));
-    }
+                               &L));
+    // 4. Y1 = LN(X + attn)
+    LnArgs ln1{ws.part, L.wo.kparts, (int)M, dm, bo_eff, desc->dtype, cur_res, resid_dtype, L.ln1_g, L.ln1_b, ln_eps,
+               y1a, split ? y1r : nullptr, nullptr, part_dtype_of(desc->dtype)};
+    ln1.ts = trace_slot(ET_K_LN1);
+    ET_TRY(layernorm_run(ln1, st));
     // 5. U = act(Y1 W1'^T + b1)
     GemmArgs f1{};
     f1.X = y1a;

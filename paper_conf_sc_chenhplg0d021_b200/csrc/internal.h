@@ -74,17 +74,7 @@ struct GemmArgs {
   int ldy;
   et_epilogue epi;
   unsigned long long* ts;   // trace slot or nullptr
-  // kEpiLN (fused residual + LayerNorm, internal): Y = LN(acc + b + resid) * gamma + beta
-  const void* resid;        // [M, ldy] in dtype
-  const float* gamma;
-  const float* beta;
-  float eps;
 };
-// internal epilogue id (not in the public et_epilogue): residual + LayerNorm fused into the GEMM,
-// row statistics exchanged across the cluster of CTAs sharing a token block (DSMEM)
-constexpr int kEpiLN = 16;
-// true if gemm_run can run `a` with kEpiLN (shape / dtype / piece constraints)
-bool gemm_ln_applies(const GemmArgs& a);
 et_status gemm_run(const GemmArgs& a, cudaStream_t stream);
 // FFN1 -> FFN2 in one launch when FFN1's pieces coincide with FFN2's K parts (kernels/tsgemm.cu)
 bool gemm_ffn_applies(const GemmArgs& f1, const GemmArgs& f2);

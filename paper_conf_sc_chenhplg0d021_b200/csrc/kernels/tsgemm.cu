@@ -133,12 +133,6 @@ struct Params {
   int ldy;
   long long part_stride;   // elements between split-K partial outputs (fp32 epilogue)
   unsigned long long* ts;  // trace slot or nullptr
-  // kEpiLN: residual [M, ldy] (operand dtype), LayerNorm parameters, CTAs per cluster (= pieces)
-  const uint8_t* resid;
-  const float* gamma;
-  const float* beta;
-  float eps;
-  int cluster_n;
 };
 
 struct __align__(16) Barriers {
@@ -160,23 +154,12 @@ struct __align__(16) Barriers {
 
 // Per epilogue: staging per epilogue warp (32 rows x 32 columns: 128 B rows in FP32, 64 B in 16-bit)
 // and as many ring slots as the rest of the 227 KB allows (9 with FP32 staging, 11 with 16-bit).
-// kEpiLN: no per-round staging; instead a stash of the FP32 pre-LN values of up to kLnMaxRows tile
-// rows (one 16 KB block of 128 tokens x 32 features per accumulator pair) and the row statistics
-// (this CTA's 4 partial sums, and one (mean, M2) per token from every CTA of the cluster); the
-// normalised output is staged in the (then idle) ring for the TMA stores.
-constexpr int kLnMaxRows = 12;
-constexpr int kLnMaxCluster = 8;
-struct LnStats {
-  float2 part[4][128];                 // per epilogue group: (mean, M2) of a token over the group's pairs
-  float2 in[kLnMaxCluster][128];       // (mean, M2) of each CTA of the cluster, written over DSMEM
-  alignas(16) float gamma[kLnMaxRows * 16], beta[kLnMaxRows * 16];   // this CTA's features
-};
+// (Round 1's O-projection + LayerNorm fused over a 4-CTA cluster with an FP32 stash measured 12.2 us
+// against 11.5 us unfused and was removed in round 2.)
 template <int kEpi> struct Smem {
-  static constexpr bool kLN = kEpi == kEpiLN;
   static constexpr size_t kStageWarp = kEpi == ET_EPI_F32 ? 4096 : 2048;
-  static constexpr size_t kStash = (size_t)(kLnMaxRows / 2) * 16384;
-  static constexpr size_t kStage = kLN ? kStash + sizeof(LnStats) : (size_t)Roles<kEpi>::EW * kStageWarp;
-  static constexpr int kSlots = kLN ? 6 : (kEpi == ET_EPI_F32 ? 9 : 11);
+  static constexpr size_t kStage = (size_t)Roles<kEpi>::EW * kStageWarp;
+  static constexpr int kSlots = kEpi == ET_EPI_F32 ? 9 : 11;
   static constexpr size_t kRing = (size_t)kSlots * kSlotBytes;
   static constexpr size_t kBytes = 1024 + kRing + kStage + sizeof(Barriers);
   static_assert(kBytes <= 232448, "shared memory budget");
@@ -231,10 +214,9 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
   uint8_t* sStage = smem + SM::kRing;
   Barriers& bar = *reinterpret_cast<Barriers*>(smem + SM::kRing + SM::kStage);
 
-  constexpr bool kLN = kEpi == kEpiLN;
 
   constexpr int kMmaWarps = Roles<kEpi>::MW, kEpiGroups = Roles<kEpi>::EG, kEpiWarps = Roles<kEpi>::EW;
-  constexpr int kWarpP = Roles<kEpi>::WP, kFillSets = kWarpP / 4, kThreads = Roles<kEpi>::threads;
+  constexpr int kWarpP = Roles<kEpi>::WP, kFillSets = kWarpP / 4;
   constexpr int kAPW = kAcc / kMmaWarps;   // accumulators per MMA warp
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -326,7 +308,6 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
   tc_fence_after();
   const uint32_t tbase = bar.tmem_base;
   if (threadIdx.x == 0) ET_TL(1);
-  if constexpr (kLN) cluster_arrive_relaxed();   // phase A: this CTA runs (DSMEM targets exist)
   // end of local row t's tiles (part A's last row ends before the padding to part B's first chunk)
   auto rend = [&](int t) { return t == rowsA - 1 ? min(bar.a_end, bar.rptr[t + 1]) : bar.rptr[t + 1]; };
 
@@ -507,13 +488,6 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
         const float2 f = unpack2<kBF16>(bsrc ? __ldg(bsrc + (size_t)row * 8 + (i & 7)) : 0u);
         *reinterpret_cast<float2*>(&bar.bias_f[2 * i]) = f;
       }
-      if constexpr (kLN) {
-        LnStats& ls0 = *reinterpret_cast<LnStats*>(sStage + SM::kStash);
-        for (int i = ew * 32 + lane; i < nrows * 16; i += kEpiWarps * 32) {
-          ls0.gamma[i] = __ldg(p.gamma + pc.i0 * 16 + i);
-          ls0.beta[i] = __ldg(p.beta + pc.i0 * 16 + i);
-        }
-      }
       named_bar_sync(1, kEpiWarps * 32);
     }
     const int g = ew >> 2;
@@ -522,20 +496,11 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
     // Per round: wait for the group's 2 accumulators (rows 8k + 2g + a), read their 32 columns with
     // one TMEM load, release them to the MMA warps, THEN do the bias / activation / store math (so
     // an MMA warp never waits for another row's epilogue arithmetic).
-    float ln_n = 0.f, ln_mean = 0.f, ln_m2 = 0.f;   // kLN: running (n, mean, M2) of this thread's values
     for (int jp = g, it = 0; jp < npairs_all; jp += kEpiGroups, ++it) {
       const int k = jp >> 2, pidx = jp & 3;   // round, pair within the round (accumulators 2p, 2p+1)
       const int t0 = 2 * jp;                  // first row of the pair
       const int na = min(2, nrows - t0);
       uint32_t r[32];
-      uint4 res4[4];
-      if constexpr (kLN) {   // residual of this thread's token and the pair's 32 features, loaded early
-        const int tok = quarter * 32 + lane;
-        const int row = min(m0 + tok, p.M - 1);
-        const uint4* rp4 = reinterpret_cast<const uint4*>(p.resid + ((size_t)row * p.ldy + (pc.i0 + t0) * 16) * 2);
-#pragma unroll
-        for (int ch = 0; ch < 4; ++ch) res4[ch] = __ldg(rp4 + ch);
-      }
       (void)k;
       GEMM_HANDOFF_WAIT(&bar.slot_full[jp], 0);   // single-use: both rows' MMAs complete
       if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it);
@@ -592,39 +557,6 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
         }
       }
       if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it + 2);
-      if constexpr (kLN) {
-        // + residual; the pair's (mean, M2) merged into this thread's running statistics (Chan et
-        // al.'s pairwise update); the FP32 pre-LN values go to the stash until the cluster's row
-        // statistics are known
-        const int tok = quarter * 32 + lane;
-#pragma unroll
-        for (int ch = 0; ch < 4; ++ch) {
-          const uint32_t w[4] = {res4[ch].x, res4[ch].y, res4[ch].z, res4[ch].w};
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const float2 f = unpack2<kBF16>(w[i]);
-            v[ch * 8 + 2 * i] += f.x;
-            v[ch * 8 + 2 * i + 1] += f.y;
-          }
-        }
-        float s1 = 0.f;
-#pragma unroll
-        for (int i = 0; i < 32; ++i) s1 += v[i];
-        const float mb = s1 * (1.0f / 32.0f);
-        float m2b = 0.f;
-#pragma unroll
-        for (int i = 0; i < 32; ++i) m2b = fmaf(v[i] - mb, v[i] - mb, m2b);
-        const float nn = ln_n + 32.f, dd = mb - ln_mean;
-        ln_mean += dd * (32.f / nn);
-        ln_m2 += m2b + dd * dd * (ln_n * 32.f / nn);
-        ln_n = nn;
-        uint8_t* sp = sStage + (size_t)(t0 >> 1) * 16384 + tok * 128;
-#pragma unroll
-        for (int ch = 0; ch < 8; ++ch)
-          *reinterpret_cast<float4*>(sp + ((ch ^ (tok & 7)) << 4)) =
-              make_float4(v[4 * ch], v[4 * ch + 1], v[4 * ch + 2], v[4 * ch + 3]);
-        continue;
-      }
       // store: registers -> this warp's 32-row staging tile -> one TMA tensor store (clipped at M by
       // the tensor map).  fp32: 128-byte rows, SWIZZLE_128B (unit c of row r at c ^ (r % 8));
       // 16-bit: 64-byte rows, SWIZZLE_64B (unit c of row r at c ^ ((r / 2) % 4)); both conflict-free.
@@ -632,7 +564,7 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
       const int col0 = t0 < rowsA ? sa.out_col + (pc.i0 + t0) * 16 : sb.out_col + (t0 - rowsA) * 16;
       const int row0 = m0 + quarter * 32;
 #ifdef ET_GEMM_DIRECT_ST
-      constexpr bool kDirect = !kLN;
+      constexpr bool kDirect = true;
 #else
       constexpr bool kDirect = false;
 #endif
@@ -689,94 +621,7 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tmap_x, const CUten
       }
       if (quarter == 0 && lane == 0 && it < 8 && g < 4) ET_TL(208 + 40 * g + 5 * it + 3);
     }
-    if constexpr (kLN) {
-      // ===== fused residual + LayerNorm (biased variance, reading C-11).  The
-      // token's d features are spread over the cluster's CTAs (one piece of nrows tile rows each):
-      // the 4 groups' statistics are merged per token, sent to every CTA of the cluster over DSMEM,
-      // merged there, and every thread normalises the pairs it computed.
-      LnStats& ls = *reinterpret_cast<LnStats*>(sStage + SM::kStash);
-      const int tok = quarter * 32 + lane;
-      const int npairs = nrows >> 1;
-      auto merge = [](float& n, float& m, float& M2, float nb, float mb, float M2b) {
-        if (nb == 0.f) return;
-        const float nn = n + nb, d = mb - m;
-        m += d * (nb / nn);
-        M2 += M2b + d * d * (n * nb / nn);
-        n = nn;
-      };
-      ls.part[g][tok] = make_float2(ln_mean, ln_m2);
-      if (ew == 0 && lane == 0) ET_TL(480);
-      named_bar_sync(1, kEpiWarps * 32);
-      if (ew == 0 && lane == 0) ET_TL(481);
-      float cn = 0.f, cm = 0.f, cM2 = 0.f;
-      if (g == 0) {
-        for (int q = 0; q < 4; ++q) {
-          const float nq = 32.f * (float)max(0, (npairs - q + 3) / 4);   // group q's pairs: q, q+4, ...
-          const float2 stq = ls.part[q][tok];
-          merge(cn, cm, cM2, nq, stq.x, stq.y);
-        }
-      }
-      cluster_wait();   // phase A: every CTA of the cluster is running
-      if (ew == 0 && lane == 0) ET_TL(483);
-      if (g == 0) {
-        const uint32_t la = smem_u32(&ls.in[cluster_ctarank()][tok]);
-        for (int r2 = 0; r2 < p.cluster_n; ++r2) st_cluster_f32x2(mapa_shared(la, (uint32_t)r2), cm, cM2);
-      }
-      cluster_arrive();   // phase B: this CTA's statistics are in every peer
-      cluster_wait();
-      if (ew == 0 && lane == 0) ET_TL(484);
-      float n = 0.f, mean = 0.f, M2 = 0.f;
-      const float nc = (float)(nrows * 16);   // equal pieces: every CTA holds nrows * 16 features
-      for (int r2 = 0; r2 < p.cluster_n; ++r2) {
-        const float2 st2 = ls.in[r2][tok];
-        merge(n, mean, M2, nc, st2.x, st2.y);
-      }
-      const float rstd = rsqrtf(M2 / n + p.eps);
-      // normalise this thread's pairs (pp = g, g + 4, ...) into the ring (idle now: every MMA
-      // completed) as the output map's boxes (32 tokens x 32 features, SWIZZLE_64B); the warp owns
-      // whole boxes (its 32 tokens), so it stores them itself
-      const int rr = lane;
-      if (ew == 0 && lane == 0) ET_TL(486);
-      for (int pp = g; pp < npairs; pp += 4) {
-        const uint8_t* sp = sStage + (size_t)pp * 16384 + tok * 128;
-        uint8_t* bx = ring + (size_t)(pp * 4 + quarter) * 2048 + rr * 64;
-        const float4* g4 = reinterpret_cast<const float4*>(&ls.gamma[pp * 32]);
-        const float4* b4 = reinterpret_cast<const float4*>(&ls.beta[pp * 32]);
-#pragma unroll
-        for (int ch = 0; ch < 4; ++ch) {
-          const float4 xa = *reinterpret_cast<const float4*>(sp + (((2 * ch) ^ (tok & 7)) << 4));
-          const float4 xb = *reinterpret_cast<const float4*>(sp + (((2 * ch + 1) ^ (tok & 7)) << 4));
-          const float4 ga = g4[2 * ch], gb = g4[2 * ch + 1], ba = b4[2 * ch], bb = b4[2 * ch + 1];
-          *reinterpret_cast<uint4*>(bx + ((ch ^ ((rr >> 1) & 3)) << 4)) = make_uint4(
-              pack2<kBF16>((xa.x - mean) * rstd * ga.x + ba.x, (xa.y - mean) * rstd * ga.y + ba.y),
-              pack2<kBF16>((xa.z - mean) * rstd * ga.z + ba.z, (xa.w - mean) * rstd * ga.w + ba.w),
-              pack2<kBF16>((xb.x - mean) * rstd * gb.x + bb.x, (xb.y - mean) * rstd * gb.y + bb.y),
-              pack2<kBF16>((xb.z - mean) * rstd * gb.z + bb.z, (xb.w - mean) * rstd * gb.w + bb.w));
-        }
-      }
-      if (ew == 0 && lane == 0) ET_TL(487);
-      fence_proxy_async_smem();
-      __syncwarp();
-      if (lane == 0) {
-        for (int pp = g; pp < npairs; pp += 4) {
-          tma_store_2d(&tmap_y, ring + (size_t)(pp * 4 + quarter) * 2048, (pc.i0 + 2 * pp) * 16, m0 + quarter * 32);
-          bulk_commit_group();
-        }
-      }
-      if (ew == 0 && lane == 0) ET_TL(485);
-      named_bar_arrive(2, kThreads);   // release the parked MMA / load warps
-    }
   }
-  if constexpr (kLN) {
-    if (warp < kMmaWarps || warp == kWarpP) {   // MMA / load warps: take part in both cluster phases,
-      __syncwarp();                             // parked on a CTA barrier (not polling the cluster
-      cluster_wait();                           // barrier) until the epilogue has normalised
-      cluster_arrive();
-      named_bar_sync(2, kThreads);
-      cluster_wait();
-    }
-  }
-
   if (warp >= kMmaWarps && warp < kWarpP && lane == 0) bulk_wait_group<0>();   // epilogue stores done
   __syncwarp();   // the producer warp: lane 0 ran the loop alone; reconverge before the block barrier
   tc_fence_before();
@@ -862,7 +707,7 @@ EncodeTiledFn get_encode() {
 
 template <int kEpi, bool kBF16>
 et_status launch_typed(const CUtensorMap& tm, const CUtensorMap& tmy, const Params& prm, dim3 grid,
-                       cudaStream_t stream, unsigned cluster_x = 0) {
+                       cudaStream_t stream) {
   auto kern = tsgemm_kernel<kEpi, kBF16>;
   static std::once_flag once;
   static cudaError_t attr_err = cudaSuccess;
@@ -870,10 +715,7 @@ et_status launch_typed(const CUtensorMap& tm, const CUtensorMap& tmy, const Para
     attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Smem<kEpi>::kBytes);
   });
   ET_CUDA(attr_err);
-  if (cluster_x > 0)
-    ET_CUDA(launch_pdl_cluster(kern, grid, dim3(Roles<kEpi>::threads), Smem<kEpi>::kBytes, stream, cluster_x, tm, tmy, prm));
-  else
-    ET_CUDA(launch_pdl(kern, grid, dim3(Roles<kEpi>::threads), Smem<kEpi>::kBytes, stream, tm, tmy, prm));
+  ET_CUDA(launch_pdl(kern, grid, dim3(Roles<kEpi>::threads), Smem<kEpi>::kBytes, stream, tm, tmy, prm));
   count_launch();
   return ET_OK;
 }
@@ -952,32 +794,6 @@ et_status make_tmap_3d_ld(CUtensorMap* tm, void* base, et_dtype dtype, uint64_t 
   return ET_OK;
 }
 
-// kEpiLN plan: np equal pieces of R tile rows (R even, R <= kLnMaxRows, np <= kLnMaxCluster), the
-// np pieces of a token block forming one cluster; the largest np whose grid fits one wave.
-// OFF unless built with -DET_GEMM_LN_FUSE: measured on C3 (profiles/r01/README.md, v4) the fused
-// O-projection + LayerNorm takes 12.2 us against 6.0 + 5.5 us unfused — the 6-slot ring (the FP32
-// stash takes the rest of shared memory) delays the first MMA by ~1.5k cycles, the cluster's
-// slowest CTA gates the statistics exchange, and the tail (stats, DSMEM exchange, normalisation)
-// costs ~8k cycles; parity is green either way (tests run both).
-static int ln_pieces(const GemmArgs& a) {
-  if (a.epi != kEpiLN || (a.dtype != ET_FP16 && a.dtype != ET_BF16) || a.nseg != 1 || a.K > 768 ||
-      !a.resid || !a.gamma || !a.beta || a.seg[0].out_col != 0 || a.ldy != a.seg[0].tile_rows * 16 ||
-      (a.ldy * 2) % 16 || !aligned16(a.resid))
-    return 0;
-#ifndef ET_GEMM_LN_FUSE
-  return 0;   // experiment (compile-time switch, off): slower than GEMM + LayerNorm kernel, see below
-#endif
-  const int rows = a.seg[0].tile_rows, mblocks = (a.M + 127) / 128;
-  int best = 0;
-  for (int np = 1; np <= kLnMaxCluster; ++np) {
-    if (rows % np || (rows / np) % 2 || rows / np > kLnMaxRows) continue;
-    if (best == 0 || mblocks * np <= 148) best = np;   // smallest valid, raised while one wave holds
-  }
-  return best;
-}
-
-bool gemm_ln_applies(const GemmArgs& a) { return ln_pieces(a) > 0; }
-
 // Launch plan of one tile GEMM: parameters, tensor maps and grid.  force_pieces > 0 replaces the
 // piece planner with that many equal tile-row pieces of the (single) segment (the FFN fusion needs
 // FFN1's pieces to coincide with FFN2's K parts).  *np_out = 0: nothing to launch (M == 0).
@@ -988,9 +804,6 @@ static et_status build_gemm(const GemmArgs& a, Params& prm, CUtensorMap& tm, CUt
   if (!aligned16(a.X) || (a.ldx * 2) % 16 || (a.k0 * 2) % 16)
     return fail(ET_ERR_INVALID_ARG, "tile GEMM: X must be 16-byte aligned with 16-byte row pitch");
   const int kparts = (a.K + 767) / 768;
-  const bool ln = a.epi == (et_epilogue)kEpiLN;
-  const int ln_np = ln ? ln_pieces(a) : 0;
-  if (ln && ln_np == 0) return fail(ET_ERR_UNSUPPORTED, "tile GEMM: fused LayerNorm epilogue does not apply");
   if (kparts > 1 && a.epi != ET_EPI_F32 && a.epi != ET_EPI_PART16)
     return fail(ET_ERR_UNSUPPORTED, "tile GEMM: K > 768 needs a partial-sum (split-K) epilogue");
   if (a.M <= 0) return ET_OK;
@@ -1029,18 +842,13 @@ static et_status build_gemm(const GemmArgs& a, Params& prm, CUtensorMap& tm, CUt
     prm.seg[s].apply_scale = gs.apply_scale;
   }
   const int kt = std::min(a.K, 768) / 16;   // tile columns per K part (bound on tiles per row)
-  prm.resid = static_cast<const uint8_t*>(a.resid);
-  prm.gamma = a.gamma;
-  prm.beta = a.beta;
-  prm.eps = a.eps;
-  prm.cluster_n = ln_np;
   const int max_rows = is_partial(a.epi) ? kMaxRows : kMaxBiasRows;
   auto fits = [&](int rows) { return rows <= max_rows && (long long)rows * kt + kChunkTiles <= (long long)kMaxBChunks * kChunkTiles; };
   int np = 0;
   // Output-contiguous segments (Q|K|V): plan the pieces over the concatenated tile rows, so the CTA
   // count is set by the total rows rather than rounded per segment (4 pieces of 36 rows instead of
   // 3 of 48 for BERT-base); a piece may straddle one segment boundary.
-  bool contiguous = a.nseg > 1 && !ln;
+  bool contiguous = a.nseg > 1;
   for (int s = 1; s < a.nseg; ++s)
     contiguous = contiguous && a.seg[s].out_col == a.seg[s - 1].out_col + a.seg[s - 1].tile_rows * 16;
   if (contiguous) {
@@ -1080,14 +888,6 @@ static et_status build_gemm(const GemmArgs& a, Params& prm, CUtensorMap& tm, CUt
     const int R = a.seg[0].tile_rows / force_pieces;
     np = 0;
     for (int k = 0; k < force_pieces; ++k) {
-      prm.piece[np].seg = prm.piece[np].seg1 = 0;
-      prm.piece[np].i0 = (int16_t)(k * R);
-      prm.piece[np].i1 = (int16_t)((k + 1) * R);
-      ++np;
-    }
-  } else if (ln) {
-    const int R = a.seg[0].tile_rows / ln_np;
-    for (int k = 0; k < ln_np; ++k) {
       prm.piece[np].seg = prm.piece[np].seg1 = 0;
       prm.piece[np].i0 = (int16_t)(k * R);
       prm.piece[np].i1 = (int16_t)((k + 1) * R);
@@ -1146,8 +946,6 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
   int np = 0;
   ET_TRY(build_gemm(a, prm, tm, tmy, grid, 0, &np));
   if (np == 0) return ET_OK;
-  const bool ln = a.epi == (et_epilogue)kEpiLN;
-  const int ln_np = ln ? ln_pieces(a) : 0;
   const bool bf = a.dtype == ET_BF16;
   switch ((int)a.epi) {
     case ET_EPI_BIAS: return bf ? launch_typed<ET_EPI_BIAS, true>(tm, tmy, prm, grid, stream)
@@ -1162,8 +960,6 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
                                : launch_typed<ET_EPI_F32, false>(tm, tmy, prm, grid, stream);
     case ET_EPI_PART16: return bf ? launch_typed<ET_EPI_PART16, true>(tm, tmy, prm, grid, stream)
                                   : launch_typed<ET_EPI_PART16, false>(tm, tmy, prm, grid, stream);
-    case kEpiLN: return bf ? launch_typed<kEpiLN, true>(tm, tmy, prm, grid, stream, (unsigned)ln_np)
-                                        : launch_typed<kEpiLN, false>(tm, tmy, prm, grid, stream, (unsigned)ln_np);
     default: break;
   }
   return fail(ET_ERR_INVALID_ARG, "tile GEMM: bad epilogue %d", (int)a.epi);
