@@ -967,14 +967,16 @@ et_status gemm_run(const GemmArgs& a, cudaStream_t stream) {
 
 // FFN1 -> FFN2 in one launch (tsgemm_ffn_kernel).  Applies when FFN1 has one segment with K <= 768
 // and a 16-bit bias + activation epilogue, FFN2 writes 16-bit split-K partial planes over K = FFN1's
-// output width, and FFN1 split into FFN2's K parts (768 output columns = 48 tile rows each) fills one
-// wave of the GPU with every CTA holding a full 48-row piece (C3: 4 pieces x 32 token blocks).
+// output width, and FFN1 split into FFN2's K parts (768 output columns = 48 tile rows each) gives at
+// least 96 CTAs (C3: 4 pieces x 32 token blocks; C4 / C5: many waves).
 bool gemm_ffn_applies(const GemmArgs& f1, const GemmArgs& f2) {
   if (f1.dtype == ET_FP32 || f1.dtype != f2.dtype || f1.nseg != 1 || f2.nseg != 1 || f1.M != f2.M) return false;
   if (f1.K > 768 || (f1.epi != ET_EPI_BIAS_GELU && f1.epi != ET_EPI_BIAS_RELU) || f2.epi != ET_EPI_PART16) return false;
   if (f2.X != f1.Y || f2.ldx != f1.ldy || f2.k0 != 0 || f2.K != f1.seg[0].tile_rows * 16 || f2.K % 768) return false;
   const int kparts = f2.K / 768, mblocks = (f1.M + 127) / 128;
-  return kparts * mblocks <= 148 && kparts * mblocks >= 96 && f1.seg[0].tile_rows == kparts * 48;
+  // no upper bound: the phases of a CTA depend on nothing outside it, so any number of waves works
+  // (and there U_c is read back while still in L2 instead of after the whole U left it)
+  return kparts * mblocks >= 96 && f1.seg[0].tile_rows == kparts * 48;
 }
 
 et_status gemm_ffn_run(const GemmArgs& f1, const GemmArgs& f2, cudaStream_t stream) {
